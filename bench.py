@@ -1,0 +1,272 @@
+#!/usr/bin/env python3
+"""Benchmark of the Owl hot path on B200: trace records/s into A-DCFG + leak tests (BASELINE.json metric).
+
+A step = one pass of the whole hot path over the workload: fold + Myers-merge every
+run of both input classes into E_fix and E_rnd (owl_build_adcfg), diff them (owl_diff_adcfg) and run the
+kernel / KS leak tests with localization (owl_leak_test).  Records are generated on the device (untimed)
+and stay resident in HBM; the workload (44.5 GB at N=1) is far larger than the 126 MB L2, so no flush is
+needed between steps.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config 2] [--impl ours|reference]
+
+Prints ONE JSON line (rank 0).  Multi-GPU: one process per GPU (torchrun), runs sharded across ranks
+(weak scaling: every rank holds the same number of runs of both classes), one key-hash exchange of the
+partial evidences (NCCL all_to_all_single), owner-side KS tests, leak rows gathered to rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "trace records/sec into A-DCFG + leak tests at 1/2/4/8 B200; % HBM peak"
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            pk = json.load(f)
+        return float(pk["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, burst copy)"
+    except Exception:  # noqa: BLE001
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index=0):
+        self.index, self.rows, self.proc = index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:  # noqa: BLE001
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 7:
+                self.rows.append(parts)
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:  # noqa: BLE001
+            self.proc.kill()
+        sm = sorted(float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit())
+        mx = max((float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()), default=None)
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower() == "active"})
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": mx, "reasons": reasons,
+                "samples": len(self.rows)}
+
+
+def _dist():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def _class_runs(p, runs, cls):
+    import tracegen
+    return [r for r in runs if tracegen.run_class(p, r) == cls]
+
+
+def cpu_baseline(cfg: int, target_s: float = 15.0):
+    """The oracle as it stands on the host cores, on a bounded sample of the same workload."""
+    import tracegen
+    from oracle import oracle
+    threads = os.cpu_count() or 1
+    div = {1: 1, 2: 16, 3: 8, 4: 64, 5: 16}[cfg]
+    runs = 2
+    while True:
+        p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=runs, runs_rnd=runs)
+        segs, _ = oracle.run_config(p, threads=threads)
+        n = sum(len(s.records) for c in (0, 1) for s in segs[c])
+        t0 = time.perf_counter()
+        f, r = oracle.build(segs[0], threads), oracle.build(segs[1], threads)
+        oracle.diff(f, r)
+        oracle.leak_test(f, r, 0.05)
+        dt = time.perf_counter() - t0
+        if dt >= target_s / 4 or runs >= 64:
+            break
+        runs = min(64, max(runs * 2, int(runs * target_s / max(dt, 1e-3) / 2)))
+    return {"value": n / dt, "unit": "records/s", "cores": threads, "kind": "oracle",
+            "sample": f"config C{cfg} grid_div={div} runs={2 * runs} ({n} records, {dt:.1f} s, build E_fix+E_rnd+diff+leak test)"}
+
+
+def run_reference(args):
+    world, rank, _ = _dist()
+    if rank != 0:
+        return
+    import tracegen
+    from oracle import oracle
+    threads = os.cpu_count() or 1
+    cfg = args.config
+    div = {1: 1, 2: 32, 3: 16, 4: 128, 5: 32}[cfg]
+    p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=2, runs_rnd=2)
+    segs, _ = oracle.run_config(p, threads=threads)
+    n = sum(len(s.records) for c in (0, 1) for s in segs[c])
+
+    def step():
+        f, r = oracle.build(segs[0], threads), oracle.build(segs[1], threads)
+        oracle.diff(f, r)
+        oracle.leak_test(f, r, 0.05)
+
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    dt = (time.perf_counter() - t0) / args.steps
+    v = n / dt
+    sample = f"config C{cfg} grid_div={div}, 2+2 runs ({n} records) per step"
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "records/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": {"workload": tracegen.CONFIG_NAMES[cfg], "sample": sample},
+        "cpu_baseline": {"value": v, "unit": "records/s", "cores": threads, "kind": "oracle", "sample": sample},
+        "e2e": {"value": v, "unit": "records/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import tracegen
+    from paper_conf_dsn_zhaoxcqzj24_b200 import api
+
+    world, rank, local = _dist()
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    cfg = args.config
+    base = tracegen.Params.preset(cfg)
+    # weak scaling: each rank holds the full per-GPU workload's runs (global run ids are disjoint)
+    rpr = base.n_runs
+    p = tracegen.Params.preset(cfg, runs_fix=base.runs_fix * world, runs_rnd=base.runs_rnd * world)
+    my_runs = list(range(rank * rpr, (rank + 1) * rpr))
+    if args.runs:
+        my_runs = my_runs[: args.runs]
+    ctx = api.Context(local)
+    stream = torch.cuda.current_stream(dev)
+    segs = []
+    t_gen = time.perf_counter()
+    for r in my_runs:
+        for m in tracegen.run_segments(p, r):
+            buf, n = tracegen.device_records(p, r, m.seq, device=dev, stream=stream)
+            segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, n))
+    torch.cuda.synchronize()
+    t_gen = time.perf_counter() - t_gen
+    n_records = sum(s.n_records for s in segs)
+    ctx.ingest(segs, stream)
+    rf, rr = _class_runs(p, my_runs, 0), _class_runs(p, my_runs, 1)
+
+    out = {}
+
+    def step():
+        ef, er = ctx.build(rf), ctx.build(rr)
+        d = ctx.diff(ef, er)
+        lk = ctx.leak_test(ef, er, 0.05)
+        out.update(n_diff=len(d), n_leaks=len(lk), info_f=ef.info(), info_r=er.info())
+        ef.destroy()
+        er.destroy()
+
+    for _ in range(args.warmup):
+        step()
+    ctx.reset_stats()
+    clocks = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ck = clocks.stop()
+    ms = e0.elapsed_time(e1) / args.steps
+    st = ctx.stats()
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    total_records = n_records * world
+    value = total_records / (ms / 1e3)
+    peak, peak_src = _peaks()
+    fold_ms = st["total_fold_ms"] / max(1, st["fold_launches"])
+    fold_bytes = 16.0 * st["total_fold_records"] / max(1, st["fold_launches"])
+    achieved = fold_bytes / (fold_ms / 1e3) / 1e9
+    res = {
+        "metric": METRIC, "value": value, "unit": "records/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": {"workload": tracegen.CONFIG_NAMES[cfg], "runs_per_gpu": len(my_runs),
+                   "records_per_gpu": n_records, "bytes_per_gpu": 16 * n_records,
+                   "l2": "inputs (%.1f GB) >> 126 MB L2; no flush needed" % (16 * n_records / 1e9),
+                   "parallelism": f"dp{world} (runs sharded, key-hash exchange)" if world > 1 else "single GPU",
+                   "generate_s_untimed": round(t_gen, 2)},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                     "traffic": None, "kernel": "fold_kernel",
+                     "note": f"16 B/record algorithmic; {st['fold_launches']} fold launches, "
+                             f"{fold_ms:.2f} ms avg (CUDA events on the launch stream); peak {peak_src}"},
+        "clocks": ck,
+        "gpu_launches": None,
+        "fold_share_of_step": (st["total_fold_ms"] / args.steps) / ms,
+        "result": {"n_diff_rows": out.get("n_diff"), "n_leaks": out.get("n_leaks"),
+                   "cells_fix": out.get("info_f", {}).get("n_cells"), "cells_rnd": out.get("info_r", {}).get("n_cells")},
+    }
+    if rank == 0 and not args.no_cpu:
+        res["cpu_baseline"] = cpu_baseline(cfg, args.cpu_seconds)
+    if rank == 0:
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=2, help="workload C1..C5 (default: configs[1], C2)")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--runs", type=int, default=0, help="limit runs per GPU (debug)")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    args = ap.parse_args()
+    import __graft_entry__
+    __graft_entry__.build_native()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -216,6 +216,13 @@ owl_status owl_absorb_evidence(owl_ctx* ctx, const owl_adcfg* like, const void* 
 owl_status owl_register_remote_runs(owl_ctx* ctx, const uint32_t* runs, const uint32_t* classes,
                                     const uint32_t* seq_len, const uint64_t* kernel_ids, size_t n_runs);
 
+/* ---- measurement ---------------------------------------------------------------------------------
+ * Fold-kernel statistics of the context: launches, the duration of the last fold launch measured with
+ * CUDA events on the context stream, and the records it folded (plus running totals). */
+owl_status owl_get_stats(const owl_ctx* ctx, uint64_t* fold_launches, double* last_fold_ms, uint64_t* last_fold_records,
+                         double* total_fold_ms, uint64_t* total_fold_records);
+owl_status owl_reset_stats(owl_ctx* ctx);
+
 void owl_free(void* host_ptr);       /* frees rows / leaks / blobs allocated by the library */
 const char* owl_last_error(void);    /* thread-local message for the last non-OK status      */
 const char* owl_version(void);

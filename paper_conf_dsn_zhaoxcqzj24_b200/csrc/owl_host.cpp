@@ -1,0 +1,895 @@
+/*
+ * owl_host.cpp — the C ABI of libowl (include/owl.h): context and segment registry (A1), Myers slot
+ * assignment and evidence bookkeeping (A4), build orchestration with capacity regrowth,
+ * canonical export, diff (A5), the kernel-leak test and leak localization (A7) around
+ * the KS kernels (A6), and the multi-GPU partition / absorb entry points.  Every step that touches records
+ * or cells runs in the CUDA kernels of owl_fold.cu / owl_tables.cu / owl_ks.cu / owl_exchange.cu; this
+ * file only marshals, schedules and sorts small host arrays.
+ */
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <string>
+#include <tuple>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "owl.h"
+#include "owl_internal.h"
+#include "owl_myers.h"
+
+#define OWL_API extern "C" __attribute__((visibility("default")))
+
+namespace {
+
+thread_local std::string g_err;
+
+owl_status fail(owl_status s, const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return s;
+}
+
+owl_status cuda_fail(cudaError_t e, const char* what) {
+  if (e == cudaErrorMemoryAllocation) return fail(OWL_ERR_OUT_OF_MEMORY, "%s: out of device memory", what);
+  return fail(OWL_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define CUDA_TRY(expr, what)                  \
+  do {                                        \
+    cudaError_t _e = (expr);                  \
+    if (_e != cudaSuccess) return cuda_fail(_e, what); \
+  } while (0)
+
+uint64_t next_pow2(uint64_t v) {
+  uint64_t p = 1;
+  while (p < v) p <<= 1;
+  return p;
+}
+
+struct RemoteRun {
+  uint32_t cls;
+  std::vector<uint64_t> kids;
+};
+
+}  // namespace
+
+struct owl_ctx {
+  int device = 0;
+  int n_sm = 148;
+  cudaStream_t stream = nullptr;
+  owl_config cfg{};
+  std::map<std::pair<uint32_t, uint32_t>, owl_segment> segs; /* (run, seq) -> segment */
+  std::map<uint32_t, RemoteRun> remote;
+  FoldStatus* d_status = nullptr;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  uint64_t cap_hint[T_NUM] = {0, 0, 0, 0};
+  /* stats */
+  uint64_t fold_launches = 0;
+  double last_fold_ms = 0;
+  uint64_t last_fold_records = 0;
+  double total_fold_ms = 0;
+  uint64_t total_fold_records = 0;
+};
+
+/* The evidence's slot list: ordered slot ids, kernel id and invocation count per slot id. */
+struct SlotState {
+  std::vector<uint32_t> order;
+  std::vector<uint64_t> kid, count;
+  uint32_t n_runs = 0;
+};
+
+struct owl_adcfg {
+  owl_ctx* ctx = nullptr;
+  uint32_t cls = 0;
+  int64_t max_run = -1;
+  SlotState slots;
+  DevTable tab[T_NUM] = {};
+  SortedTable sorted[T_NUM];
+  bool sorted_ok = false;
+  uint64_t n_records = 0;
+  ExchangeCell* send = nullptr;
+  ~owl_adcfg() {
+    for (int t = 0; t < T_NUM; ++t) {
+      owl_table_free(&tab[t]);
+      owl_sorted_free(&sorted[t]);
+    }
+    if (send) cudaFree(send);
+  }
+};
+
+namespace {
+
+/* A4: merge one run's kernel sequence into the slot list with Myers; returns the slot of
+   each of the run's invocations (in seq order). */
+std::vector<uint32_t> slot_merge(SlotState& s, const std::vector<uint32_t>& seqs, const std::vector<uint64_t>& kids) {
+  std::vector<uint32_t> out(seqs.size());
+  if (s.n_runs == 0) { /* the first run: slots are its invocation indices */
+    uint32_t mx = 0;
+    for (uint32_t q : seqs) mx = std::max(mx, q + 1);
+    s.kid.assign(mx, 0);
+    s.count.assign(mx, 0);
+    for (size_t i = 0; i < seqs.size(); ++i) {
+      s.kid[seqs[i]] = kids[i];
+      s.count[seqs[i]] = 1;
+      s.order.push_back(seqs[i]);
+      out[i] = seqs[i];
+    }
+    s.n_runs = 1;
+    return out;
+  }
+  std::vector<uint64_t> a;
+  for (uint32_t sl : s.order) a.push_back(s.kid[sl]);
+  std::vector<OwlEdit> ops = owl_myers(a, kids);
+  std::vector<uint32_t> order;
+  for (const OwlEdit& o : ops) {
+    if (o.op == OWL_EDIT_MATCH) {
+      const uint32_t sl = s.order[o.i];
+      s.count[sl] += 1;
+      out[o.j] = sl;
+      order.push_back(sl);
+    } else if (o.op == OWL_EDIT_DEL) {
+      order.push_back(s.order[o.i]);
+    } else {
+      const uint32_t sl = (uint32_t)s.kid.size();
+      s.kid.push_back(kids[o.j]);
+      s.count.push_back(1);
+      out[o.j] = sl;
+      order.push_back(sl);
+    }
+  }
+  s.order.swap(order);
+  s.n_runs += 1;
+  return out;
+}
+
+struct PlannedSeg {
+  owl_segment s;
+  uint32_t slot;
+};
+
+/* Gathers runs, checks classes, assigns slots.  Runs must be ascending and above `after`. */
+owl_status plan_runs(owl_ctx* ctx, const uint32_t* runs, size_t n_runs, int64_t after, uint32_t* cls_io,
+                     bool cls_known, SlotState& ss, std::vector<PlannedSeg>& plan) {
+  std::vector<uint32_t> rs(runs, runs + n_runs);
+  std::sort(rs.begin(), rs.end());
+  for (size_t i = 1; i < rs.size(); ++i)
+    if (rs[i] == rs[i - 1]) return fail(OWL_ERR_INVALID_ARG, "run %u listed twice", rs[i]);
+  if (!rs.empty() && (int64_t)rs[0] <= after)
+    return fail(OWL_ERR_INVALID_ARG, "run %u is not above the runs already merged (%lld)", rs[0], (long long)after);
+  for (uint32_t r : rs) {
+    auto lo = ctx->segs.lower_bound({r, 0});
+    std::vector<uint32_t> seqs;
+    std::vector<uint64_t> kids;
+    std::vector<const owl_segment*> local;
+    uint32_t cls = 0;
+    bool have = false;
+    for (auto it = lo; it != ctx->segs.end() && it->first.first == r; ++it) {
+      seqs.push_back(it->first.second);
+      kids.push_back(it->second.kernel_id);
+      local.push_back(&it->second);
+      cls = it->second.input_class;
+      have = true;
+    }
+    if (!have) {
+      auto rm = ctx->remote.find(r);
+      if (rm == ctx->remote.end()) return fail(OWL_ERR_STATE, "run %u has not been ingested", r);
+      cls = rm->second.cls;
+      kids = rm->second.kids;
+      for (size_t q = 0; q < kids.size(); ++q) seqs.push_back((uint32_t)q);
+    }
+    if (!cls_known) { *cls_io = cls; cls_known = true; }
+    if (cls != *cls_io)
+      return fail(OWL_ERR_INVALID_ARG, "run %u has input class %u, expected %u (one class per evidence)", r, cls, *cls_io);
+    std::vector<uint32_t> sl = slot_merge(ss, seqs, kids);
+    for (size_t q = 0; q < local.size(); ++q) plan.push_back({*local[q], sl[q]});
+  }
+  if (ss.kid.size() > OWL_MAX_SLOT)
+    return fail(OWL_ERR_CAPACITY, "%zu evidence slots exceed the limit %u", ss.kid.size(), OWL_MAX_SLOT);
+  return OWL_OK;
+}
+
+const char* kerr_text(uint32_t code) {
+  switch (code) {
+    case KERR_GWARP: return "gwarp >= n_warps";
+    case KERR_BBFIELDS: return "non-zero addr/lane/ins on a BB_ENTRY";
+    case KERR_MTYPE: return "unknown memory type";
+    case KERR_NOBB: return "MEM record before the warp's first BB_ENTRY";
+    case KERR_BBMISMATCH: return "MEM record bb != the warp's current BB";
+    default: return "?";
+  }
+}
+
+/* One fold pass over the planned segments into `tab` (A1-A3).  Returns OWL_OK, or an error; sets
+   *overflow to the bitmask of tables that must grow. */
+owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable* tab, unsigned* overflow,
+                     uint64_t* n_records) {
+  const cudaStream_t st = ctx->stream;
+  *overflow = 0;
+  const uint32_t tile_shift = 14;
+  std::vector<FoldSeg> fs(plan.size());
+  std::vector<void*> scratch;
+  std::vector<uint64_t*> perms(plan.size(), nullptr);
+  uint64_t seen_words = 0, tiles = 0, nrec = 0;
+  for (size_t i = 0; i < plan.size(); ++i) seen_words += (plan[i].s.n_warps + 31) / 32;
+  uint32_t* seen = (uint32_t*)owl_dev_alloc((seen_words + 1) * 4);
+  if (!seen) return fail(OWL_ERR_OUT_OF_MEMORY, "fold: warp bitmap");
+  scratch.push_back(seen);
+  CUDA_TRY(cudaMemsetAsync(seen, 0, (seen_words + 1) * 4, st), "fold: memset");
+  uint64_t so = 0;
+  owl_status status = OWL_OK;
+  for (size_t i = 0; i < plan.size() && status == OWL_OK; ++i) {
+    const owl_segment& s = plan[i].s;
+    const uint4* rec = (const uint4*)s.records;
+    if (s.n_records && (s.flags & OWL_SEG_HOST_RECORDS)) { /* stage host records into HBM */
+      uint4* d = (uint4*)owl_dev_alloc(s.n_records * 16);
+      if (!d) { status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: staging %llu records", (unsigned long long)s.n_records); break; }
+      scratch.push_back(d);
+      cudaError_t e = cudaMemcpyAsync(d, s.records, s.n_records * 16, cudaMemcpyHostToDevice, st);
+      if (e != cudaSuccess) { status = cuda_fail(e, "fold: H2D"); break; }
+      rec = d;
+    }
+    if (s.n_records && !(s.flags & OWL_SEG_WARP_MAJOR)) { /* channel order: stable bucket by warp (R17) */
+      uint4* d = (uint4*)owl_dev_alloc(s.n_records * 16);
+      uint64_t* perm = (uint64_t*)owl_dev_alloc(s.n_records * 8);
+      if (!d || !perm) { owl_dev_free(d); owl_dev_free(perm); status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: bucketing"); break; }
+      scratch.push_back(d);
+      scratch.push_back(perm);
+      cudaError_t e = owl_bucket_by_warp(rec, s.n_records, s.n_warps, d, perm, st);
+      if (e != cudaSuccess) { status = cuda_fail(e, "fold: bucketing"); break; }
+      rec = d;
+      perms[i] = perm;
+    }
+    fs[i].rec = rec;
+    fs[i].n = s.n_records;
+    fs[i].tile0 = tiles;
+    fs[i].slot = plan[i].slot;
+    fs[i].n_warps = s.n_warps;
+    fs[i].seen = seen + so;
+    fs[i].seg_index = (uint32_t)i;
+    fs[i]._pad = 0;
+    so += (s.n_warps + 31) / 32;
+    tiles += (s.n_records + (1ull << tile_shift) - 1) >> tile_shift;
+    nrec += s.n_records;
+  }
+  FoldSeg* dsegs = nullptr;
+  if (status == OWL_OK) {
+    dsegs = (FoldSeg*)owl_dev_alloc(fs.size() * sizeof(FoldSeg) + 16);
+    if (!dsegs) status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: segment table");
+  }
+  FoldStatus hs;
+  if (status == OWL_OK) {
+    scratch.push_back(dsegs);
+    cudaMemcpyAsync(dsegs, fs.data(), fs.size() * sizeof(FoldSeg), cudaMemcpyHostToDevice, st);
+    hs.first_error = ~0ull;
+    hs.not_warp_major = ~0ull;
+    hs.overflow = 0;
+    hs.limit = 0;
+    hs.tile_counter = 0;
+    cudaMemcpyAsync(ctx->d_status, &hs, sizeof hs, cudaMemcpyHostToDevice, st);
+    FoldArgs a;
+    a.segs = dsegs;
+    a.n_segs = (uint32_t)fs.size();
+    a.tile_shift = tile_shift;
+    a.n_tiles = tiles;
+    for (int t = 0; t < T_NUM; ++t) a.tab[t] = tab[t];
+    a.status = ctx->d_status;
+    const int per_sm = ctx->cfg.fold_ctas_per_sm ? (int)ctx->cfg.fold_ctas_per_sm : owl_fold_ctas_per_sm();
+    cudaEventRecord(ctx->ev0, st);
+    cudaError_t e = tiles ? owl_launch_fold(a, ctx->n_sm * per_sm, st) : cudaSuccess;
+    cudaEventRecord(ctx->ev1, st);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&hs, ctx->d_status, sizeof hs, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) status = cuda_fail(e, "fold kernel");
+    else {
+      float ms = 0;
+      cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1);
+      if (tiles) ctx->fold_launches += 1;
+      ctx->last_fold_ms = ms;
+      ctx->last_fold_records = nrec;
+      ctx->total_fold_ms += ms;
+      ctx->total_fold_records += nrec;
+    }
+  }
+  if (status == OWL_OK) {
+    if (hs.first_error != ~0ull) {
+      const uint32_t si = (uint32_t)(hs.first_error >> 40);
+      uint64_t idx = (hs.first_error >> 3) & ((1ull << 37) - 1);
+      const uint32_t code = (uint32_t)(hs.first_error & 7);
+      if (si < plan.size() && perms[si]) { /* map back to the caller's record index */
+        uint64_t orig = idx;
+        cudaMemcpy(&orig, perms[si] + idx, 8, cudaMemcpyDeviceToHost);
+        idx = orig;
+      }
+      status = fail(OWL_ERR_MALFORMED_TRACE, "malformed trace: run %u seq %u record %llu: %s",
+                    si < plan.size() ? plan[si].s.run : 0, si < plan.size() ? plan[si].s.seq : 0,
+                    (unsigned long long)idx, kerr_text(code));
+    } else if (hs.not_warp_major != ~0ull) {
+      const uint32_t si = (uint32_t)(hs.not_warp_major >> 32);
+      status = fail(OWL_ERR_INVALID_ARG,
+                    "segment (run %u, seq %u) is flagged OWL_SEG_WARP_MAJOR but warp %u's records are not contiguous",
+                    plan[si].s.run, plan[si].s.seq, (uint32_t)hs.not_warp_major);
+    } else if (hs.limit) {
+      status = fail(OWL_ERR_CAPACITY, (hs.limit & 2) ? "a traced warp visits more than 256 distinct basic blocks"
+                                                     : "a basic-block visit ordinal j exceeds 2^22-1");
+    }
+    *overflow = hs.overflow;
+  }
+  for (void* p : scratch) owl_dev_free(p);
+  *n_records = nrec;
+  return status;
+}
+
+uint64_t default_cap(owl_ctx* ctx, int t) {
+  if (ctx->cap_hint[t]) return ctx->cap_hint[t];
+  if (t == T_ADDR) return ctx->cfg.addr_capacity ? next_pow2(ctx->cfg.addr_capacity) : (1ull << 22);
+  return ctx->cfg.cf_capacity ? next_pow2(ctx->cfg.cf_capacity) : (1ull << 14);
+}
+
+/* Builds fresh tables for the planned segments, regrowing on overflow. */
+owl_status build_tables(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable* tab, uint64_t* n_records) {
+  uint64_t cap[T_NUM];
+  for (int t = 0; t < T_NUM; ++t) cap[t] = default_cap(ctx, t);
+  const uint32_t max_regrow = ctx->cfg.max_regrow ? ctx->cfg.max_regrow : 6;
+  for (uint32_t attempt = 0;; ++attempt) {
+    for (int t = 0; t < T_NUM; ++t) {
+      cudaError_t e = owl_table_alloc(&tab[t], cap[t], ctx->stream);
+      if (e != cudaSuccess) {
+        for (int u = 0; u <= t; ++u) owl_table_free(&tab[u]);
+        return cuda_fail(e, "table allocation");
+      }
+    }
+    unsigned overflow = 0;
+    owl_status s = fold_pass(ctx, plan, tab, &overflow, n_records);
+    if (s != OWL_OK) {
+      for (int t = 0; t < T_NUM; ++t) owl_table_free(&tab[t]);
+      return s;
+    }
+    if (!overflow) {
+      for (int t = 0; t < T_NUM; ++t) ctx->cap_hint[t] = std::max(ctx->cap_hint[t], cap[t]);
+      return OWL_OK;
+    }
+    for (int t = 0; t < T_NUM; ++t) owl_table_free(&tab[t]);
+    if (attempt >= max_regrow) return fail(OWL_ERR_CAPACITY, "A-DCFG tables still full after %u regrowths", attempt);
+    for (int t = 0; t < T_NUM; ++t)
+      if (overflow & (1u << t)) cap[t] *= 4;
+  }
+}
+
+owl_status ensure_sorted(owl_adcfg* g) {
+  if (g->sorted_ok) return OWL_OK;
+  for (int t = 0; t < T_NUM; ++t) {
+    owl_sorted_free(&g->sorted[t]);
+    cudaError_t e = owl_table_sorted(g->tab[t], &g->sorted[t], g->ctx->stream);
+    if (e != cudaSuccess) return cuda_fail(e, "canonical sort");
+  }
+  g->sorted_ok = true;
+  return OWL_OK;
+}
+
+/* Merges the cells of `src` (sorted) into g's tables, rebuilding them with room for both. */
+owl_status merge_into(owl_adcfg* g, SortedTable* src) {
+  owl_status s = ensure_sorted(g);
+  if (s != OWL_OK) return s;
+  cudaStream_t st = g->ctx->stream;
+  for (int t = 0; t < T_NUM; ++t) {
+    const uint64_t need = g->sorted[t].n + src[t].n;
+    uint64_t cap = std::max<uint64_t>(g->tab[t].cap, next_pow2(2 * need + 16));
+    DevTable nt{};
+    CUDA_TRY(owl_table_alloc(&nt, cap, st), "merge: table allocation");
+    CUDA_TRY(cudaMemsetAsync(g->ctx->d_status, 0, sizeof(FoldStatus), st), "merge");
+    CUDA_TRY(owl_table_insert_sorted(nt, t, g->sorted[t].k, g->sorted[t].c, g->sorted[t].n, g->ctx->d_status, st), "merge");
+    CUDA_TRY(owl_table_insert_sorted(nt, t, src[t].k, src[t].c, src[t].n, g->ctx->d_status, st), "merge");
+    CUDA_TRY(cudaStreamSynchronize(st), "merge");
+    owl_table_free(&g->tab[t]);
+    g->tab[t] = nt;
+  }
+  g->sorted_ok = false;
+  return OWL_OK;
+}
+
+template <class T>
+T* host_copy(const std::vector<T>& v) {
+  T* p = (T*)malloc(sizeof(T) * (v.size() ? v.size() : 1));
+  if (p && !v.empty()) memcpy(p, v.data(), sizeof(T) * v.size());
+  return p;
+}
+
+/* unpack canonical keys into row fields */
+void unpack(int t, const Key128& k, uint32_t& slot, uint32_t& a, uint32_t& b, uint32_t& c, uint64_t& x) {
+  if (t == T_ADDR) {
+    slot = (uint32_t)(k.hi >> 48);
+    a = (uint32_t)((k.hi >> 30) & 0x3FFFFu); /* bb */
+    b = (uint32_t)((k.hi >> 22) & 0xFFu);    /* ins */
+    c = (uint32_t)(k.hi & OWL_MAX_J);        /* j */
+    x = k.lo;
+  } else {
+    slot = (uint32_t)(k.hi >> 32);
+    a = (uint32_t)k.hi; /* bb or src */
+    b = (uint32_t)(k.lo >> 32);
+    c = (uint32_t)k.lo;
+    x = 0;
+  }
+}
+
+}  // namespace
+
+/* ================================== ABI ================================== */
+
+OWL_API const char* owl_last_error(void) { return g_err.c_str(); }
+OWL_API const char* owl_version(void) { return "owl-b200 0.1 (sm_100a)"; }
+OWL_API void owl_free(void* p) { free(p); }
+
+OWL_API owl_status owl_ctx_create(int cuda_device, owl_ctx** out) {
+  if (!out) return fail(OWL_ERR_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  int n = 0;
+  cudaError_t e = cudaGetDeviceCount(&n);
+  if (e != cudaSuccess || n == 0) return fail(OWL_ERR_CUDA, "no CUDA device: %s", cudaGetErrorString(e));
+  if (cuda_device < 0 || cuda_device >= n) return fail(OWL_ERR_INVALID_ARG, "device %d out of range", cuda_device);
+  CUDA_TRY(cudaSetDevice(cuda_device), "cudaSetDevice");
+  cudaDeviceProp prop;
+  CUDA_TRY(cudaGetDeviceProperties(&prop, cuda_device), "cudaGetDeviceProperties");
+  if (prop.major < 10) return fail(OWL_ERR_CUDA, "device %d is sm_%d%d; libowl is built for sm_100a", cuda_device, prop.major, prop.minor);
+  owl_ctx* c = new owl_ctx();
+  c->device = cuda_device;
+  c->n_sm = prop.multiProcessorCount;
+  c->d_status = (FoldStatus*)owl_dev_alloc(sizeof(FoldStatus));
+  if (!c->d_status) { delete c; return fail(OWL_ERR_OUT_OF_MEMORY, "status"); }
+  cudaEventCreate(&c->ev0);
+  cudaEventCreate(&c->ev1);
+  *out = c;
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_ctx_destroy(owl_ctx* ctx) {
+  if (!ctx) return OWL_OK;
+  cudaSetDevice(ctx->device);
+  owl_dev_free(ctx->d_status);
+  if (ctx->ev0) cudaEventDestroy(ctx->ev0);
+  if (ctx->ev1) cudaEventDestroy(ctx->ev1);
+  delete ctx;
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_ctx_set_config(owl_ctx* ctx, const owl_config* cfg) {
+  if (!ctx) return fail(OWL_ERR_INVALID_ARG, "ctx is NULL");
+  if (cfg) ctx->cfg = *cfg;
+  else ctx->cfg = owl_config{};
+  for (int t = 0; t < T_NUM; ++t) ctx->cap_hint[t] = 0;
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_ingest_traces(owl_ctx* ctx, const owl_segment* segs, size_t n_segs, owl_stream_t stream) {
+  if (!ctx || (!segs && n_segs)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  for (size_t i = 0; i < n_segs; ++i) {
+    const owl_segment& s = segs[i];
+    if (s.n_records && !s.records) return fail(OWL_ERR_INVALID_ARG, "segment %zu: records is NULL", i);
+    if (s.input_class > 1) return fail(OWL_ERR_INVALID_ARG, "segment %zu: input_class %u", i, s.input_class);
+    if (((uintptr_t)s.records & 15) != 0) return fail(OWL_ERR_INVALID_ARG, "segment %zu: records not 16-byte aligned", i);
+    if (ctx->segs.count({s.run, s.seq})) return fail(OWL_ERR_INVALID_ARG, "segment (run %u, seq %u) already ingested", s.run, s.seq);
+    auto lo = ctx->segs.lower_bound({s.run, 0});
+    if (lo != ctx->segs.end() && lo->first.first == s.run && lo->second.input_class != s.input_class)
+      return fail(OWL_ERR_INVALID_ARG, "run %u: segments of different input classes", s.run);
+    for (size_t j = 0; j < i; ++j)
+      if (segs[j].run == s.run && segs[j].seq == s.seq) return fail(OWL_ERR_INVALID_ARG, "segment (run %u, seq %u) twice", s.run, s.seq);
+  }
+  for (size_t i = 0; i < n_segs; ++i) ctx->segs[{segs[i].run, segs[i].seq}] = segs[i];
+  ctx->stream = (cudaStream_t)stream;
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_forget_runs(owl_ctx* ctx, const uint32_t* runs, size_t n_runs) {
+  if (!ctx || (!runs && n_runs)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  for (size_t i = 0; i < n_runs; ++i) {
+    auto lo = ctx->segs.lower_bound({runs[i], 0});
+    while (lo != ctx->segs.end() && lo->first.first == runs[i]) lo = ctx->segs.erase(lo);
+    ctx->remote.erase(runs[i]);
+  }
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_register_remote_runs(owl_ctx* ctx, const uint32_t* runs, const uint32_t* classes,
+                                            const uint32_t* seq_len, const uint64_t* kernel_ids, size_t n_runs) {
+  if (!ctx || (n_runs && (!runs || !classes || !seq_len))) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  size_t off = 0;
+  for (size_t i = 0; i < n_runs; ++i) {
+    RemoteRun rr;
+    rr.cls = classes[i];
+    rr.kids.assign(kernel_ids + off, kernel_ids + off + seq_len[i]);
+    off += seq_len[i];
+    ctx->remote[runs[i]] = rr;
+  }
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_build_adcfg(owl_ctx* ctx, const uint32_t* runs, size_t n_runs, owl_adcfg** out) {
+  if (!ctx || !out || (!runs && n_runs)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  *out = nullptr;
+  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+  owl_adcfg* g = new owl_adcfg();
+  g->ctx = ctx;
+  std::vector<PlannedSeg> plan;
+  owl_status s = plan_runs(ctx, runs, n_runs, -1, &g->cls, false, g->slots, plan);
+  if (s == OWL_OK) s = build_tables(ctx, plan, g->tab, &g->n_records);
+  if (s != OWL_OK) { delete g; return s; }
+  for (size_t i = 0; i < n_runs; ++i) g->max_run = std::max<int64_t>(g->max_run, runs[i]);
+  *out = g;
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_adcfg_accumulate(owl_ctx* ctx, owl_adcfg* g, const uint32_t* runs, size_t n_runs) {
+  if (!ctx || !g || (!runs && n_runs)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  if (!n_runs) return OWL_OK;
+  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+  SlotState ss = g->slots;
+  std::vector<PlannedSeg> plan;
+  uint32_t cls = g->cls;
+  owl_status s = plan_runs(ctx, runs, n_runs, g->max_run, &cls, g->slots.n_runs > 0, ss, plan);
+  if (s != OWL_OK) return s;
+  owl_adcfg tmp;
+  tmp.ctx = ctx;
+  uint64_t nrec = 0;
+  s = build_tables(ctx, plan, tmp.tab, &nrec);
+  if (s == OWL_OK) s = ensure_sorted(&tmp);
+  if (s == OWL_OK) s = merge_into(g, tmp.sorted);
+  if (s != OWL_OK) return s;
+  g->slots = ss;
+  g->cls = cls;
+  g->n_records += nrec;
+  for (size_t i = 0; i < n_runs; ++i) g->max_run = std::max<int64_t>(g->max_run, runs[i]);
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_adcfg_info_get(const owl_adcfg* g, owl_adcfg_info* info) {
+  if (!g || !info) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  owl_status s = ensure_sorted(const_cast<owl_adcfg*>(g));
+  if (s != OWL_OK) return s;
+  info->input_class = g->cls;
+  info->n_runs = g->slots.n_runs;
+  info->n_slots = (uint32_t)g->slots.order.size();
+  info->_pad = 0;
+  for (int t = 0; t < T_NUM; ++t) info->n_cells[t] = g->sorted[t].n;
+  info->n_records = g->n_records;
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_adcfg_destroy(owl_adcfg* g) {
+  if (g) {
+    cudaSetDevice(g->ctx->device);
+    delete g;
+  }
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_adcfg_export(const owl_adcfg* gc, const char* path, void** host_blob, size_t* bytes) {
+  if (!gc) return fail(OWL_ERR_INVALID_ARG, "NULL adcfg");
+  owl_adcfg* g = const_cast<owl_adcfg*>(gc);
+  CUDA_TRY(cudaSetDevice(g->ctx->device), "cudaSetDevice");
+  owl_status s = ensure_sorted(g);
+  if (s != OWL_OK) return s;
+  std::vector<Key128> k[T_NUM];
+  std::vector<unsigned long long> c[T_NUM];
+  for (int t = 0; t < T_NUM; ++t) {
+    k[t].resize(g->sorted[t].n);
+    c[t].resize(g->sorted[t].n);
+    if (g->sorted[t].n) {
+      CUDA_TRY(cudaMemcpy(k[t].data(), g->sorted[t].k, g->sorted[t].n * sizeof(Key128), cudaMemcpyDeviceToHost), "export");
+      CUDA_TRY(cudaMemcpy(c[t].data(), g->sorted[t].c, g->sorted[t].n * 8, cudaMemcpyDeviceToHost), "export");
+    }
+  }
+  std::vector<unsigned char> out;
+  auto put = [&](const void* p, size_t n) { const unsigned char* q = (const unsigned char*)p; out.insert(out.end(), q, q + n); };
+  auto u32 = [&](uint32_t v) { put(&v, 4); };
+  auto u64 = [&](uint64_t v) { put(&v, 8); };
+  size_t need = 56 + g->slots.order.size() * 24 + k[0].size() * 16 + k[1].size() * 24 + k[2].size() * 24 + k[3].size() * 32;
+  out.reserve(need);
+  put("OWLADCFG", 8);
+  u32(1);
+  u32(g->cls);
+  u32(g->slots.n_runs);
+  u32((uint32_t)g->slots.order.size());
+  for (int t = 0; t < T_NUM; ++t) u64(k[t].size());
+  for (uint32_t sl : g->slots.order) { u32(sl); u32(0); u64(g->slots.kid[sl]); u64(g->slots.count[sl]); }
+  for (int t = 0; t < T_NUM; ++t)
+    for (size_t i = 0; i < k[t].size(); ++i) {
+      uint32_t slot, a, b, cc;
+      uint64_t x;
+      unpack(t, k[t][i], slot, a, b, cc, x);
+      if (t == T_NODE) { u32(slot); u32(a); }
+      else if (t == T_EDGE) { u32(slot); u32(a); u32(cc); u32(0); }
+      else if (t == T_TRIPLE) { u32(slot); u32(a); u32(b); u32(cc); }
+      else { u32(slot); u32(a); u32(b); u32(cc); u64(x); }
+      u64(c[t][i]);
+    }
+  if (path) {
+    FILE* f = fopen(path, "wb");
+    if (!f) return fail(OWL_ERR_INVALID_ARG, "cannot open %s", path);
+    size_t w = fwrite(out.data(), 1, out.size(), f);
+    fclose(f);
+    if (w != out.size()) return fail(OWL_ERR_INVALID_ARG, "short write to %s", path);
+  }
+  if (host_blob) {
+    *host_blob = host_copy(out);
+    if (!*host_blob) return fail(OWL_ERR_OUT_OF_MEMORY, "export blob");
+  }
+  if (bytes) *bytes = out.size();
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_diff_adcfg(owl_ctx* ctx, const owl_adcfg* a, const owl_adcfg* b, owl_diff** rows, size_t* n_rows) {
+  if (!ctx || !a || !b || !rows || !n_rows) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+  owl_adcfg* ga = const_cast<owl_adcfg*>(a);
+  owl_adcfg* gb = const_cast<owl_adcfg*>(b);
+  owl_status s = ensure_sorted(ga);
+  if (s == OWL_OK) s = ensure_sorted(gb);
+  if (s != OWL_OK) return s;
+  std::vector<owl_diff> out;
+  const uint32_t NA = 0xFFFFFFFFu;
+  for (int t = 0; t < T_NUM; ++t) {
+    std::vector<DiffCell> d;
+    CUDA_TRY(owl_diff_sorted(ga->sorted[t], gb->sorted[t], d, ctx->stream), "diff");
+    for (const DiffCell& c : d) {
+      owl_diff r;
+      uint32_t slot, x1, x2, x3;
+      uint64_t x;
+      unpack(t, c.k, slot, x1, x2, x3, x);
+      r.table = (uint32_t)t;
+      r.slot = slot;
+      r.bb = r.ins = r.j = r.prev = r.next = NA;
+      r._pad = 0;
+      r.x = 0;
+      if (t == T_NODE) r.bb = x1;
+      else if (t == T_EDGE) { r.prev = x1; r.next = x3; }
+      else if (t == T_TRIPLE) { r.bb = x1; r.prev = x2; r.next = x3; }
+      else { r.bb = x1; r.ins = x2; r.j = x3; r.x = x; }
+      r.count_a = c.ca;
+      r.count_b = c.cb;
+      out.push_back(r);
+    }
+  }
+  /* slot table: (slot, kernel_id) -> invocation count */
+  std::map<std::pair<uint32_t, uint64_t>, uint64_t> sa, sb;
+  for (uint32_t sl : ga->slots.order) sa[{sl, ga->slots.kid[sl]}] = ga->slots.count[sl];
+  for (uint32_t sl : gb->slots.order) sb[{sl, gb->slots.kid[sl]}] = gb->slots.count[sl];
+  std::map<std::pair<uint32_t, uint64_t>, std::pair<uint64_t, uint64_t>> all;
+  for (auto& e : sa) all[e.first].first = e.second;
+  for (auto& e : sb) all[e.first].second = e.second;
+  for (auto& e : all)
+    if (e.second.first != e.second.second) {
+      owl_diff r;
+      r.table = OWL_TABLE_SLOT;
+      r.slot = e.first.first;
+      r.bb = r.ins = r.j = r.prev = r.next = NA;
+      r._pad = 0;
+      r.x = e.first.second;
+      r.count_a = e.second.first;
+      r.count_b = e.second.second;
+      out.push_back(r);
+    }
+  *rows = host_copy(out);
+  *n_rows = out.size();
+  return *rows ? OWL_OK : fail(OWL_ERR_OUT_OF_MEMORY, "diff rows");
+}
+
+namespace {
+
+struct Alignment {
+  std::vector<OwlEdit> ops;
+  std::vector<uint32_t> f2r;   /* fix slot -> rnd slot (UINT32_MAX if unaligned) */
+  std::vector<int> pos_of_f;   /* fix slot -> script position */
+};
+
+Alignment align(const owl_adcfg* f, const owl_adcfg* r) {
+  Alignment al;
+  std::vector<uint64_t> a, b;
+  for (uint32_t s : f->slots.order) a.push_back(f->slots.kid[s]);
+  for (uint32_t s : r->slots.order) b.push_back(r->slots.kid[s]);
+  al.ops = owl_myers(a, b);
+  al.f2r.assign(f->slots.kid.size(), 0xFFFFFFFFu);
+  al.pos_of_f.assign(f->slots.kid.size(), -1);
+  for (size_t p = 0; p < al.ops.size(); ++p)
+    if (al.ops[p].op == OWL_EDIT_MATCH) {
+      const uint32_t sf = f->slots.order[al.ops[p].i];
+      al.f2r[sf] = r->slots.order[al.ops[p].j];
+      al.pos_of_f[sf] = (int)p;
+    }
+  return al;
+}
+
+owl_status run_ks(owl_ctx* ctx, const owl_adcfg* f, const owl_adcfg* r, double sig, const Alignment& al,
+                  std::vector<owl_ks_row>& rows, std::vector<int>& pos) {
+  owl_status s = ensure_sorted(const_cast<owl_adcfg*>(f));
+  if (s == OWL_OK) s = ensure_sorted(const_cast<owl_adcfg*>(r));
+  if (s != OWL_OK) return s;
+  const uint32_t NA = 0xFFFFFFFFu;
+  std::vector<std::tuple<int, uint32_t, uint32_t, uint32_t, uint32_t, size_t>> order;
+  for (int tbl : {T_TRIPLE, T_ADDR}) {
+    std::vector<KsOutRow> out;
+    CUDA_TRY(owl_ks_run(tbl, f->sorted[tbl], r->sorted[tbl], al.f2r, sig, out, ctx->stream), "KS tests");
+    for (const KsOutRow& o : out) {
+      owl_ks_row row;
+      Key128 kf{o.hi_f, 0}, kr{o.hi_r, 0};
+      uint32_t sf, sr, a1, a2, a3, b1, b2, b3;
+      uint64_t x;
+      unpack(tbl, kf, sf, a1, a2, a3, x);
+      unpack(tbl, kr, sr, b1, b2, b3, x);
+      row.kind = tbl == T_TRIPLE ? OWL_LEAK_CONTROL_FLOW : OWL_LEAK_DATA_FLOW;
+      row.slot_fix = sf;
+      row.slot_rnd = sr;
+      row.bb = a1;
+      row.ins = tbl == T_ADDR ? a2 : NA;
+      row.j = tbl == T_ADDR ? a3 : NA;
+      row.n = o.n; row.m = o.m; row.K_lo = o.K_lo; row.K_hi = o.K_hi;
+      row.D = o.D; row.p = o.p; row.fail = o.fail; row._pad = 0;
+      order.emplace_back(al.pos_of_f[sf], row.kind, row.bb, row.ins, row.j, rows.size());
+      rows.push_back(row);
+    }
+  }
+  std::sort(order.begin(), order.end());
+  std::vector<owl_ks_row> sorted;
+  pos.clear();
+  for (auto& o : order) { sorted.push_back(rows[std::get<5>(o)]); pos.push_back(std::get<0>(o)); }
+  rows.swap(sorted);
+  return OWL_OK;
+}
+
+}  // namespace
+
+OWL_API owl_status owl_ks_tests(owl_ctx* ctx, const owl_adcfg* e_fix, const owl_adcfg* e_rnd, double significance,
+                                owl_ks_row** rows, size_t* n_rows) {
+  if (!ctx || !e_fix || !e_rnd || !rows || !n_rows) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+  Alignment al = align(e_fix, e_rnd);
+  std::vector<owl_ks_row> out;
+  std::vector<int> pos;
+  owl_status s = run_ks(ctx, e_fix, e_rnd, significance, al, out, pos);
+  if (s != OWL_OK) return s;
+  *rows = host_copy(out);
+  *n_rows = out.size();
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_leak_test(owl_ctx* ctx, const owl_adcfg* f, const owl_adcfg* r, double significance,
+                                 owl_leak** leaks, size_t* n_leaks) {
+  if (!ctx || !f || !r || !leaks || !n_leaks) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+  const uint32_t NA = 0xFFFFFFFFu;
+  const double nan = std::nan("");
+  Alignment al = align(f, r);
+  std::vector<owl_leak> out;
+  /* kernel leaks: unaligned invocations, or aligned with different counts (reading R12) */
+  for (const OwlEdit& o : al.ops) {
+    owl_leak l;
+    memset(&l, 0, sizeof l);
+    l.kind = OWL_LEAK_KERNEL;
+    l.bb = l.ins = l.j = NA;
+    l.D = l.p = nan;
+    if (o.op == OWL_EDIT_DEL) {
+      const uint32_t s = f->slots.order[o.i];
+      l.slot_fix = s; l.slot_rnd = NA; l.kernel_id = f->slots.kid[s]; l.n = f->slots.count[s]; l.m = 0;
+      out.push_back(l);
+    } else if (o.op == OWL_EDIT_INS) {
+      const uint32_t s = r->slots.order[o.j];
+      l.slot_fix = NA; l.slot_rnd = s; l.kernel_id = r->slots.kid[s]; l.n = 0; l.m = r->slots.count[s];
+      out.push_back(l);
+    } else {
+      const uint32_t sf = f->slots.order[o.i], sr = r->slots.order[o.j];
+      const unsigned __int128 lhs = (unsigned __int128)f->slots.count[sf] * r->slots.n_runs;
+      const unsigned __int128 rhs = (unsigned __int128)r->slots.count[sr] * f->slots.n_runs;
+      if (lhs != rhs) {
+        l.slot_fix = sf; l.slot_rnd = sr; l.kernel_id = f->slots.kid[sf];
+        l.n = f->slots.count[sf]; l.m = r->slots.count[sr];
+        out.push_back(l);
+      }
+    }
+  }
+  std::vector<owl_ks_row> rows;
+  std::vector<int> pos;
+  owl_status s = run_ks(ctx, f, r, significance, al, rows, pos);
+  if (s != OWL_OK) return s;
+  auto to_leak = [&](const owl_ks_row& k, uint32_t kind) {
+    owl_leak l;
+    l.kind = kind; l.slot_fix = k.slot_fix; l.slot_rnd = k.slot_rnd; l.bb = k.bb;
+    l.ins = kind == OWL_LEAK_DATA_FLOW ? k.ins : NA;
+    l.j = kind == OWL_LEAK_DATA_FLOW ? k.j : NA;
+    l.kernel_id = f->slots.kid[k.slot_fix];
+    l.n = k.n; l.m = k.m; l.K_lo = k.K_lo; l.K_hi = k.K_hi; l.D = k.D; l.p = k.p;
+    return l;
+  };
+  /* CF leaks at the node's BB */
+  for (const owl_ks_row& k : rows)
+    if (k.fail && k.kind == OWL_LEAK_CONTROL_FLOW) out.push_back(to_leak(k, OWL_LEAK_CONTROL_FLOW));
+  /* DF leak at (slot, bb, ins) if any visit j fails; representative = min p, ties -> smallest j (R14) */
+  size_t i = 0;
+  while (i < rows.size()) {
+    if (rows[i].kind != OWL_LEAK_DATA_FLOW) { ++i; continue; }
+    size_t e = i;
+    int best = -1;
+    while (e < rows.size() && rows[e].kind == OWL_LEAK_DATA_FLOW && pos[e] == pos[i] && rows[e].bb == rows[i].bb &&
+           rows[e].ins == rows[i].ins) {
+      if (rows[e].fail && (best < 0 || rows[e].p < rows[best].p)) best = (int)e;
+      ++e;
+    }
+    if (best >= 0) out.push_back(to_leak(rows[best], OWL_LEAK_DATA_FLOW));
+    i = e;
+  }
+  *leaks = host_copy(out);
+  *n_leaks = out.size();
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_partition_evidence(owl_ctx* ctx, const owl_adcfg* partial, int world, void** d_send,
+                                          uint64_t* send_bytes) {
+  if (!ctx || !partial || world < 1 || !d_send || !send_bytes) return fail(OWL_ERR_INVALID_ARG, "bad argument");
+  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+  owl_adcfg* g = const_cast<owl_adcfg*>(partial);
+  owl_status s = ensure_sorted(g);
+  if (s != OWL_OK) return s;
+  if (g->send) { cudaFree(g->send); g->send = nullptr; }
+  std::vector<uint64_t> counts(world);
+  CUDA_TRY(owl_partition_cells(g->sorted, world, &g->send, counts.data(), ctx->stream), "partition");
+  for (int w = 0; w < world; ++w) send_bytes[w] = counts[w] * sizeof(ExchangeCell);
+  *d_send = g->send;
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_absorb_evidence(owl_ctx* ctx, const owl_adcfg* like, const void* d_recv, const uint64_t* recv_bytes,
+                                       int world, int rank, owl_adcfg** owned) {
+  (void)rank;
+  if (!ctx || !like || world < 1 || !owned || !recv_bytes) return fail(OWL_ERR_INVALID_ARG, "bad argument");
+  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+  uint64_t total = 0;
+  for (int w = 0; w < world; ++w) {
+    if (recv_bytes[w] % sizeof(ExchangeCell)) return fail(OWL_ERR_INVALID_ARG, "recv_bytes[%d] not a multiple of %zu", w, sizeof(ExchangeCell));
+    total += recv_bytes[w] / sizeof(ExchangeCell);
+  }
+  if (total && !d_recv) return fail(OWL_ERR_INVALID_ARG, "d_recv is NULL");
+  owl_adcfg* g = new owl_adcfg();
+  g->ctx = ctx;
+  g->cls = like->cls;
+  g->slots = like->slots;
+  g->max_run = like->max_run;
+  g->n_records = like->n_records;
+  for (int t = 0; t < T_NUM; ++t) {
+    cudaError_t e = owl_table_alloc(&g->tab[t], next_pow2(2 * total + 1024), ctx->stream);
+    if (e != cudaSuccess) { delete g; return cuda_fail(e, "absorb: tables"); }
+  }
+  cudaError_t e = cudaMemsetAsync(ctx->d_status, 0, sizeof(FoldStatus), ctx->stream);
+  if (e == cudaSuccess) e = owl_absorb_cells(g->tab, (const ExchangeCell*)d_recv, total, ctx->d_status, ctx->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+  if (e != cudaSuccess) { delete g; return cuda_fail(e, "absorb"); }
+  *owned = g;
+  return OWL_OK;
+}
+
+/* Library statistics for measurement (not part of the analysis): fold launches, last fold duration
+   (CUDA events on the context stream around the fold kernel) and records. */
+OWL_API owl_status owl_get_stats(const owl_ctx* ctx, uint64_t* fold_launches, double* last_fold_ms,
+                                 uint64_t* last_fold_records, double* total_fold_ms, uint64_t* total_fold_records) {
+  if (!ctx) return fail(OWL_ERR_INVALID_ARG, "NULL ctx");
+  if (fold_launches) *fold_launches = ctx->fold_launches;
+  if (last_fold_ms) *last_fold_ms = ctx->last_fold_ms;
+  if (last_fold_records) *last_fold_records = ctx->last_fold_records;
+  if (total_fold_ms) *total_fold_ms = ctx->total_fold_ms;
+  if (total_fold_records) *total_fold_records = ctx->total_fold_records;
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_reset_stats(owl_ctx* ctx) {
+  if (!ctx) return fail(OWL_ERR_INVALID_ARG, "NULL ctx");
+  ctx->fold_launches = 0;
+  ctx->last_fold_ms = ctx->total_fold_ms = 0;
+  ctx->last_fold_records = ctx->total_fold_records = 0;
+  return OWL_OK;
+}

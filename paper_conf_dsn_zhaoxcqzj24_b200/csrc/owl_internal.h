@@ -1,0 +1,144 @@
+/*
+ * owl_internal.h — internal declarations of libowl (CUDA kernels <-> host runtime).  Not part of the ABI.
+ *
+ * Device A-DCFG tables are open-addressing hash tables of 32-byte cells {key_hi, key_lo, count, pad}
+ * (one L2 sector per cell: probe, claim and count update touch one sector).  Keys pack the canonical
+ * key so that ascending (key_hi, key_lo) as unsigned integers IS the canonical order:
+ *   node   hi = slot<<32 | bb                         lo = 0
+ *   edge   hi = slot<<32 | src                        lo = dst
+ *   triple hi = slot<<32 | bb                         lo = prev<<32 | next
+ *   addr   hi = slot<<48 | bb<<30 | ins<<22 | j       lo = x (the full 64-bit address word)
+ * Field limits: slot < 0xFFFF, bb < 2^18 (record format), ins < 2^8, j < 2^22.  A real key never has
+ * key_hi == ~0, so (~0, ~0) marks an empty cell.
+ */
+#ifndef OWL_INTERNAL_H
+#define OWL_INTERNAL_H
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <vector>
+
+#include "owl.h"
+
+#define OWL_EMPTY_KEY 0xFFFFFFFFFFFFFFFFull
+#define OWL_MAX_SLOT 0xFFFEu
+#define OWL_MAX_J ((1u << 22) - 1u)
+#define OWL_NONE_BB 0xFFFFFFFEu /* "no basic block entered yet" */
+
+enum { T_NODE = 0, T_EDGE = 1, T_TRIPLE = 2, T_ADDR = 3, T_NUM = 4 };
+
+/* error codes written by kernels (low 3 bits of the packed error word) */
+enum {
+  KERR_NONE = 0,
+  KERR_GWARP = 1,     /* gwarp >= n_warps                                  */
+  KERR_BBFIELDS = 2,  /* BB_ENTRY with non-zero addr / lane / ins          */
+  KERR_MTYPE = 3,     /* memory type > 8                                   */
+  KERR_NOBB = 4,      /* MEM before the warp's first BB_ENTRY              */
+  KERR_BBMISMATCH = 5 /* MEM bb != the warp's current BB                   */
+};
+
+struct owl_cell {
+  unsigned long long hi, lo, count, pad;
+};
+
+struct DevTable {
+  owl_cell* cells;     /* cap cells */
+  unsigned long long* fill; /* number of claimed cells (device counter) */
+  uint64_t cap;        /* power of two */
+};
+
+/* Shared device status of one fold launch */
+struct FoldStatus {
+  unsigned long long first_error;   /* min over errors of (seg<<40 | idx<<3 | code), ~0 = none      */
+  unsigned long long not_warp_major;/* min (seg<<32 | gwarp) of a warp seen twice, ~0 = none         */
+  unsigned int overflow;            /* bitmask of tables that exceeded their load limit             */
+  unsigned int limit;               /* bitmask: 1 = slot/j field limit exceeded, 2 = visits map full */
+  unsigned long long tile_counter;  /* persistent-kernel work counter                               */
+};
+
+/* One segment as the fold kernel sees it */
+struct FoldSeg {
+  const uint4* rec;   /* 16-byte records (device) */
+  uint64_t n;         /* records */
+  uint64_t tile0;     /* first global tile index of this segment */
+  uint32_t slot;      /* evidence slot of this invocation */
+  uint32_t n_warps;
+  uint32_t* seen;     /* bitmap of n_warps bits (warp-major check), zeroed */
+  uint32_t seg_index; /* position in the build's (run, seq)-sorted segment list */
+  uint32_t _pad;
+};
+
+struct FoldArgs {
+  const FoldSeg* segs;
+  uint32_t n_segs;
+  uint32_t tile_shift;   /* tile = 1 << tile_shift records */
+  uint64_t n_tiles;
+  DevTable tab[T_NUM];
+  FoldStatus* status;
+};
+
+/* ---- launchers (owl_fold.cu, owl_tables.cu, owl_ks.cu, owl_exchange.cu) ---- */
+cudaError_t owl_launch_fold(const FoldArgs& a, int grid, cudaStream_t st);
+int owl_fold_ctas_per_sm();
+
+struct Key128 {
+  unsigned long long hi, lo;
+};
+/* A table compacted and sorted by (hi, lo): the canonical order.  Device arrays owned by the holder. */
+struct SortedTable {
+  Key128* k = nullptr;
+  unsigned long long* c = nullptr;
+  uint64_t n = 0;
+};
+
+cudaError_t owl_table_alloc(DevTable* t, uint64_t cap, cudaStream_t st);
+void owl_table_free(DevTable* t);
+cudaError_t owl_table_sorted(const DevTable& t, SortedTable* out, cudaStream_t st);
+void owl_sorted_free(SortedTable* s);
+/* inserts every cell of a sorted table into a hash table (evidence merge of partial builds / absorb) */
+cudaError_t owl_table_insert_sorted(const DevTable& t, int tbl, const Key128* k, const unsigned long long* c,
+                                    uint64_t n, FoldStatus* st_dev, cudaStream_t st);
+
+struct DiffCell {
+  Key128 k;
+  unsigned long long ca, cb;
+};
+/* full outer join of two sorted tables: the differing cells in canonical order */
+cudaError_t owl_diff_sorted(const SortedTable& a, const SortedTable& b, std::vector<DiffCell>& out, cudaStream_t st);
+
+/* stable bucketing of a segment's records by gwarp (channel-order input, reading R17) */
+cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, uint4* out, uint64_t* perm,
+                               cudaStream_t st);
+
+/* KS tests over one table kind (T_TRIPLE: H_cf per node; T_ADDR: H_addr per (bb, ins, j)) */
+struct KsOutRow {
+  unsigned long long hi_f, hi_r; /* attribute keys (fix / rnd side) */
+  unsigned long long n, m, K_lo, K_hi;
+  double D, p;
+  uint32_t fail, _pad;
+};
+cudaError_t owl_ks_run(int tbl, const SortedTable& f, const SortedTable& r, const std::vector<uint32_t>& slot_f2r,
+                       double significance, std::vector<KsOutRow>& rows, cudaStream_t st);
+
+/* multi-GPU: pack every cell of the four sorted tables by owner rank */
+struct ExchangeCell {
+  unsigned long long hi, lo, count;
+  uint32_t tbl, _pad;
+};
+cudaError_t owl_partition_cells(const SortedTable* tabs, int world, ExchangeCell** d_send, uint64_t* counts,
+                                cudaStream_t st);
+cudaError_t owl_absorb_cells(const DevTable* tabs, const ExchangeCell* cells, uint64_t n, FoldStatus* st_dev,
+                             cudaStream_t st);
+
+/* device memory helpers (owl_tables.cu) */
+void* owl_dev_alloc(size_t bytes);
+void owl_dev_free(void* p);
+
+/* host-side key helpers */
+static inline uint64_t owl_mix64(uint64_t x) {
+  x ^= x >> 33; x *= 0xff51afd7ed558ccdull; x ^= x >> 33; x *= 0xc4ceb9fe1a85ec53ull; x ^= x >> 33;
+  return x;
+}
+
+#endif

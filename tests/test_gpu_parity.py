@@ -1,0 +1,253 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded inputs.
+
+Bar (BASELINE.json north_star): canonical A-DCFG dumps (node / edge / triple / address tables,
+slot table) and diff rows bit-exact; KS K exact and D bit-identical; p within 1e-9 relative (x when p underflows);
+leak verdicts and locations identical except where p is within 1e-9 of the threshold.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import tracegen
+from oracle import oracle
+from tests import helpers as H
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+from paper_conf_dsn_zhaoxcqzj24_b200 import api  # noqa: E402
+
+SIG = 0.05
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    return api.Context(0)
+
+
+def _gpu_segments(p, runs, interleaved=False):
+    segs = []
+    for r in runs:
+        for m in tracegen.run_segments(p, r):
+            if interleaved:
+                rec = tracegen.interleave(tracegen.host_records(p, r, m.seq))
+                buf = torch.from_numpy(rec.view(np.uint8).copy()).cuda()
+                segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, len(rec), flags=0))
+            else:
+                buf, n = tracegen.device_records(p, r, m.seq)
+                segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, n))
+    return segs
+
+
+def _oracle_segments(p, runs):
+    out = {0: [], 1: []}
+    for r in runs:
+        for m in tracegen.run_segments(p, r):
+            out[m.input_class].append(oracle.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id,
+                                                     tracegen.host_records(p, r, m.seq)))
+    return out
+
+
+def _runs_of(p, cls):
+    return [r for r in range(p.n_runs) if tracegen.run_class(p, r) == cls]
+
+
+def _same_p(a, b):
+    if a == b:
+        return True
+    if a < 2.2250738585072014e-308 or b < 2.2250738585072014e-308:
+        xa, xb = -math.log(max(a, 5e-324) / 2), -math.log(max(b, 5e-324) / 2)
+        return abs(xa - xb) <= 1e-9 * max(abs(xa), abs(xb)) or (a == 0 and b == 0)
+    return abs(a - b) <= 1e-9 * max(abs(a), abs(b))
+
+
+def assert_ks_parity(g, o):
+    assert len(g) == len(o)
+    for f in ("kind", "slot_fix", "slot_rnd", "bb", "ins", "j", "n", "m", "K_lo", "K_hi"):
+        assert np.array_equal(g[f], o[f]), f
+    assert np.array_equal(g["D"].view(np.uint64), o["D"].view(np.uint64)), "D must be bit-identical"
+    for i in range(len(g)):
+        assert _same_p(float(g["p"][i]), float(o["p"][i])), (i, g["p"][i], o["p"][i])
+        if g["fail"][i] != o["fail"][i]:
+            assert abs(float(o["p"][i]) - SIG) <= 1e-9 * SIG, i
+
+
+def assert_leak_parity(g, o):
+    near = [i for i in range(len(o)) if o["kind"][i] != 0 and abs(float(o["p"][i]) - SIG) <= 1e-9 * SIG]
+    assert not near, "a p-value inside the tolerance band of the threshold: compare verdicts by hand"
+    assert len(g) == len(o)
+    for f in ("kind", "slot_fix", "slot_rnd", "bb", "ins", "j", "kernel_id", "n", "m", "K_lo", "K_hi"):
+        assert np.array_equal(g[f], o[f]), f
+    ks = g["kind"] != 0
+    assert np.array_equal(g["D"][ks].view(np.uint64), o["D"][ks].view(np.uint64))
+    for i in np.flatnonzero(ks):
+        assert _same_p(float(g["p"][i]), float(o["p"][i]))
+
+
+def _build_and_compare(ctx, p, runs=None, interleaved=False):
+    runs = list(range(p.n_runs)) if runs is None else runs
+    segs = _gpu_segments(p, runs, interleaved)
+    ctx.ingest(segs)
+    try:
+        rf = [r for r in runs if tracegen.run_class(p, r) == 0]
+        rr = [r for r in runs if tracegen.run_class(p, r) == 1]
+        ef, er = ctx.build(rf), ctx.build(rr)
+        osg = _oracle_segments(p, runs)
+        of, orr = oracle.build(osg[0]), oracle.build(osg[1])
+        bf, bo = ef.export(), of.export()
+        if bf != bo:
+            pf, po = H.parse_blob(bf), H.parse_blob(bo)
+            for t in ("slots", "node", "edge", "triple", "addr"):
+                assert len(pf[t]) == len(po[t]) and np.array_equal(pf[t], po[t]), t
+        assert bf == bo
+        assert er.export() == orr.export()
+        assert_ks_parity(ctx.ks_tests(ef, er, SIG), oracle.ks_tests(of, orr, SIG))
+        assert_leak_parity(ctx.leak_test(ef, er, SIG), oracle.leak_test(of, orr, SIG))
+        gd, od = ctx.diff(ef, er), oracle.diff(of, orr)
+        assert len(gd) == len(od) and np.array_equal(gd, od)
+        return ef, er, of, orr
+    finally:
+        ctx.forget_runs(runs)
+
+
+def test_generator_device_equals_host():
+    """T3: the counter-based generator gives byte-identical records on host and device."""
+    for cfg, div in ((1, 1), (2, 64), (3, 16), (4, 128), (5, 32)):
+        p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=1, runs_rnd=1)
+        for r in (0, 1):
+            for m in tracegen.run_segments(p, r):
+                buf, n = tracegen.device_records(p, r, m.seq)
+                host = tracegen.host_records(p, r, m.seq)
+                assert n == len(host)
+                assert bytes(buf.cpu().numpy()) == host.tobytes(), (cfg, r, m.seq)
+
+
+def test_w1(ctx):
+    doc = H.load_golden("w1.json")
+    rec = H.w1_records(doc)
+    buf = torch.from_numpy(rec.view(np.uint8).copy()).cuda()
+    ctx.ingest([api.Segment(0, 0, 0, 2, 10, buf, len(rec))])
+    try:
+        g = ctx.build([0])
+        p = H.parse_blob(g.export())
+        got = H.blob_tables_as_lists(p)
+        for t in ("node", "edge", "triple", "addr"):
+            assert got[t] == doc["expected"][t], t
+        assert g.export() == oracle.build([oracle.Segment(0, 0, 0, 2, 10, rec)]).export()
+    finally:
+        ctx.forget_runs([0])
+
+
+@pytest.mark.parametrize("variant", ["mem_before_bb", "bb_mismatch", "gwarp", "bb_fields", "mtype"])
+def test_malformed_same_report(ctx, variant):
+    rec = H.w1_records()
+    if variant == "mem_before_bb":
+        rec = np.concatenate([rec[1:2], rec[0:1], rec[2:]])
+    elif variant == "bb_mismatch":
+        rec["meta"][4] = (rec["meta"][4] & ~np.uint32(0x3FFFF << 8)) | np.uint32(2 << 8)
+    elif variant == "gwarp":
+        rec["gwarp"][10:] = 7
+    elif variant == "bb_fields":
+        rec["addr"][3] = 5
+    else:
+        rec["addr"][7] = np.uint64(12) << np.uint64(60)
+    with pytest.raises(oracle.OracleError) as eo:
+        oracle.build([oracle.Segment(0, 0, 0, 2, 10, rec)])
+    buf = torch.from_numpy(rec.view(np.uint8).copy()).cuda()
+    for flags in (api.OWL_SEG_WARP_MAJOR, 0):
+        if variant == "mem_before_bb" and flags:
+            pass
+        ctx.ingest([api.Segment(0, 0, 0, 2, 10, buf, len(rec), flags=flags)])
+        try:
+            with pytest.raises(api.OwlError, match="OWL_ERR_MALFORMED_TRACE") as eg:
+                ctx.build([0])
+            assert str(eo.value).split(": ", 1)[1] in str(eg.value), (str(eo.value), str(eg.value))
+        finally:
+            ctx.forget_runs([0])
+
+
+@pytest.mark.parametrize("cfg,div,nf,nr", [(1, 1, 10, 10), (2, 32, 3, 3), (3, 16, 2, 2), (4, 64, 2, 2), (5, 16, 3, 3)])
+def test_config_parity(ctx, cfg, div, nf, nr):
+    p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=nf, runs_rnd=nr)
+    _build_and_compare(ctx, p)
+
+
+def test_c4_kernel_leak_parity(ctx):
+    """C4 at small scale with enough RND runs that some skip the conditional kernel (Myers inserts)."""
+    p = tracegen.Params.preset(4, grid_div=256, runs_fix=3, runs_rnd=6)
+    ef, er, of, orr = _build_and_compare(ctx, p)
+    assert ef.info()["n_slots"] == 4
+
+
+@pytest.mark.parametrize("cfg,div", [(1, 1), (2, 64), (5, 32)])
+def test_channel_order_input(ctx, cfg, div):
+    """Reading R17: interleaved (channel-order) records give the identical A-DCFG."""
+    p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=2, runs_rnd=2)
+    _build_and_compare(ctx, p, interleaved=True)
+
+
+def test_accumulate_equals_single_build(ctx):
+    p = tracegen.Params.preset(4, grid_div=256, runs_fix=4, runs_rnd=4)
+    runs = list(range(p.n_runs))
+    ctx.ingest(_gpu_segments(p, runs))
+    try:
+        rr = _runs_of(p, 1)
+        whole = ctx.build(rr)
+        part = ctx.build(rr[:2])
+        part.accumulate(rr[2:])
+        assert part.export() == whole.export()
+        with pytest.raises(api.OwlError, match="INVALID_ARG"):
+            part.accumulate(rr[:1])  # runs must be merged in ascending order
+    finally:
+        ctx.forget_runs(runs)
+
+
+def test_identical_inputs_no_differences(ctx):
+    """North-star invariant: identical traces => zero diff rows, every D = 0, no leaks."""
+    p = tracegen.Params.preset(2, grid_div=64, runs_fix=3, runs_rnd=1)
+    runs = _runs_of(p, 0)
+    ctx.ingest(_gpu_segments(p, runs))
+    try:
+        a, b = ctx.build(runs), ctx.build(runs)
+        assert len(ctx.diff(a, b)) == 0
+        ks = ctx.ks_tests(a, b)
+        assert len(ks) > 0 and np.all(ks["D"] == 0.0) and np.all(ks["p"] == 2.0)
+        assert len(ctx.leak_test(a, b)) == 0
+        r0, r1 = ctx.build(runs[:1]), ctx.build(runs[1:2])  # FIX runs repeat one secret
+        assert len(ctx.diff(r0, r1)) == 0
+    finally:
+        ctx.forget_runs(runs)
+
+
+def test_capacity_regrow(ctx):
+    """A deliberately tiny initial table must regrow and still give the exact result."""
+    p = tracegen.Params.preset(2, grid_div=64, runs_fix=1, runs_rnd=1)
+    ctx.set_config(addr_capacity=1024, cf_capacity=16)
+    try:
+        _build_and_compare(ctx, p)
+    finally:
+        ctx.set_config()
+
+
+def test_full_size_c2_run_parity(ctx):
+    """configs[1] (C2, the bench workload) at full size in the bench's launch configuration: one run's
+    A-DCFG against the oracle, and E_fix over 4 FIX runs = 4 x that run (FIX repeats one secret)."""
+    p = tracegen.Params.preset(2, runs_fix=4, runs_rnd=0)
+    segs = _gpu_segments(p, [0, 1, 2, 3])
+    ctx.ingest(segs)
+    try:
+        g0 = ctx.build([0])
+        o0 = oracle.build(_oracle_segments(p, [0])[0])
+        assert g0.export() == o0.export()
+        ev = H.parse_blob(ctx.build([0, 1, 2, 3]).export())
+        one = H.parse_blob(g0.export())
+        for t in ("node", "edge", "triple", "addr"):
+            assert np.array_equal(ev[t]["count"], 4 * one[t]["count"]), t
+        n_rec = sum(s.n_records for s in segs)
+        assert int(ev["addr"]["count"].sum()) + int(ev["node"]["count"].sum()) == n_rec
+    finally:
+        ctx.forget_runs([0, 1, 2, 3])
