@@ -186,17 +186,34 @@ def run_ours(args):
     rf, rr = _class_runs(p, my_runs, 0), _class_runs(p, my_runs, 1)
 
     out = {}
+    brk = {}
+
+    def tick(name, t0):
+        if args.breakdown:
+            torch.cuda.synchronize()
+            t1 = time.perf_counter()
+            brk[name] = brk.get(name, 0.0) + (t1 - t0) * 1e3
+            return t1
+        return t0
 
     def step():
-        ef, er = ctx.build(rf), ctx.build(rr)
+        t0 = time.perf_counter()
+        ef = ctx.build(rf)
+        t0 = tick("build_fix", t0)
+        er = ctx.build(rr)
+        t0 = tick("build_rnd", t0)
         d = ctx.diff(ef, er)
+        t0 = tick("diff", t0)
         lk = ctx.leak_test(ef, er, 0.05)
+        t0 = tick("leak_test", t0)
         out.update(n_diff=len(d), n_leaks=len(lk), info_f=ef.info(), info_r=er.info())
         ef.destroy()
         er.destroy()
+        tick("destroy", t0)
 
     for _ in range(args.warmup):
         step()
+    brk.clear()
     ctx.reset_stats()
     clocks = ClockSampler(local)
     if world > 1:
@@ -238,6 +255,7 @@ def run_ours(args):
         "clocks": ck,
         "gpu_launches": None,
         "fold_share_of_step": (st["total_fold_ms"] / args.steps) / ms,
+        "breakdown_ms": {k: v / args.steps for k, v in brk.items()} if args.breakdown else None,
         "result": {"n_diff_rows": out.get("n_diff"), "n_leaks": out.get("n_leaks"),
                    "cells_fix": out.get("info_f", {}).get("n_cells"), "cells_rnd": out.get("info_r", {}).get("n_cells")},
     }
@@ -258,6 +276,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--runs", type=int, default=0, help="limit runs per GPU (debug)")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--breakdown", action="store_true", help="host-timed per-call breakdown (syncs between calls)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     args = ap.parse_args()
     import __graft_entry__

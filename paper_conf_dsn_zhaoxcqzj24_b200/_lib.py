@@ -5,7 +5,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libowl.so")
+LIB_PATH = os.environ.get("OWL_LIBOWL_PATH") or os.path.join(_HERE, "libowl.so")
 
 u32, u64, vp, sz = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_size_t
 

@@ -63,9 +63,12 @@ cudaError_t owl_partition_cells(const SortedTable* tabs, int world, ExchangeCell
   unsigned long long *dcnt = nullptr, *doff = nullptr, *dcur = nullptr;
   uint64_t total = 0;
   for (int t = 0; t < T_NUM; ++t) total += tabs[t].n;
-  if (cudaMalloc(&dcnt, world * 8) || cudaMalloc(&doff, world * 8) || cudaMalloc(&dcur, world * 8) ||
-      cudaMalloc(d_send, (total + 1) * sizeof(ExchangeCell))) {
-    cudaFree(dcnt); cudaFree(doff); cudaFree(dcur);
+  dcnt = (unsigned long long*)owl_dev_alloc(world * 8);
+  doff = (unsigned long long*)owl_dev_alloc(world * 8);
+  dcur = (unsigned long long*)owl_dev_alloc(world * 8);
+  *d_send = (ExchangeCell*)owl_dev_alloc((total + 1) * sizeof(ExchangeCell));
+  if (!dcnt || !doff || !dcur || !*d_send) {
+    owl_dev_free(dcnt); owl_dev_free(doff); owl_dev_free(dcur); owl_dev_free(*d_send);
     return cudaErrorMemoryAllocation;
   }
   cudaMemsetAsync(dcnt, 0, world * 8, st);
@@ -83,7 +86,7 @@ cudaError_t owl_partition_cells(const SortedTable* tabs, int world, ExchangeCell
       scatter_owner_kernel<<<grid_for(tabs[t].n, 256), 256, 0, st>>>(tabs[t].k, tabs[t].c, tabs[t].n, t, world, doff,
                                                                      dcur, *d_send);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  cudaFree(dcnt); cudaFree(doff); cudaFree(dcur);
+  owl_dev_free(dcnt); owl_dev_free(doff); owl_dev_free(dcur);
   return e == cudaSuccess ? cudaGetLastError() : e;
 }
 

@@ -103,7 +103,7 @@ struct owl_adcfg {
       owl_table_free(&tab[t]);
       owl_sorted_free(&sorted[t]);
     }
-    if (send) cudaFree(send);
+    if (send) owl_dev_free(send);
   }
 };
 
@@ -261,31 +261,61 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     tiles += (s.n_records + (1ull << tile_shift) - 1) >> tile_shift;
     nrec += s.n_records;
   }
+  /* run batching (owl_fold.cu): groups of up to 32 segments of one slot, ascending run */
+  std::vector<uint32_t> order(fs.size());
+  for (size_t i = 0; i < order.size(); ++i) order[i] = (uint32_t)i;
+  std::stable_sort(order.begin(), order.end(), [&](uint32_t x, uint32_t y) { return fs[x].slot < fs[y].slot; });
+  std::vector<FoldSeg> gsegs;
+  std::vector<FoldGroup> groups;
+  uint64_t items = 0;
+  for (size_t i = 0; i < order.size();) {
+    size_t e = i;
+    uint64_t npos = 0;
+    while (e < order.size() && e - i < 32 && fs[order[e]].slot == fs[order[i]].slot) {
+      npos = std::max<uint64_t>(npos, (fs[order[e]].n + (1ull << tile_shift) - 1) >> tile_shift);
+      ++e;
+    }
+    FoldGroup g;
+    g.item0 = items;
+    g.first_seg = (uint32_t)gsegs.size();
+    g.n_members = (uint32_t)(e - i);
+    for (size_t q = i; q < e; ++q) gsegs.push_back(fs[order[q]]);
+    if (npos) { groups.push_back(g); items += npos; }
+    else gsegs.resize(g.first_seg);
+    i = e;
+  }
   FoldSeg* dsegs = nullptr;
+  FoldGroup* dgroups = nullptr;
   if (status == OWL_OK) {
-    dsegs = (FoldSeg*)owl_dev_alloc(fs.size() * sizeof(FoldSeg) + 16);
-    if (!dsegs) status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: segment table");
+    dsegs = (FoldSeg*)owl_dev_alloc(gsegs.size() * sizeof(FoldSeg) + 16);
+    dgroups = (FoldGroup*)owl_dev_alloc(groups.size() * sizeof(FoldGroup) + 16);
+    if (!dsegs || !dgroups) status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: segment table");
   }
   FoldStatus hs;
   if (status == OWL_OK) {
     scratch.push_back(dsegs);
-    cudaMemcpyAsync(dsegs, fs.data(), fs.size() * sizeof(FoldSeg), cudaMemcpyHostToDevice, st);
+    scratch.push_back(dgroups);
+    cudaMemcpyAsync(dsegs, gsegs.data(), gsegs.size() * sizeof(FoldSeg), cudaMemcpyHostToDevice, st);
+    cudaMemcpyAsync(dgroups, groups.data(), groups.size() * sizeof(FoldGroup), cudaMemcpyHostToDevice, st);
     hs.first_error = ~0ull;
     hs.not_warp_major = ~0ull;
     hs.overflow = 0;
     hs.limit = 0;
     hs.tile_counter = 0;
+    hs.n_flush = hs.n_bypass = hs.n_claim = 0;
     cudaMemcpyAsync(ctx->d_status, &hs, sizeof hs, cudaMemcpyHostToDevice, st);
     FoldArgs a;
     a.segs = dsegs;
-    a.n_segs = (uint32_t)fs.size();
+    a.groups = dgroups;
+    a.n_groups = (uint32_t)groups.size();
     a.tile_shift = tile_shift;
-    a.n_tiles = tiles;
+    a.n_items = items;
     for (int t = 0; t < T_NUM; ++t) a.tab[t] = tab[t];
     a.status = ctx->d_status;
+    a.mode = getenv("OWL_FOLD_MODE") ? (uint32_t)atoi(getenv("OWL_FOLD_MODE")) : 0u;
     const int per_sm = ctx->cfg.fold_ctas_per_sm ? (int)ctx->cfg.fold_ctas_per_sm : owl_fold_ctas_per_sm();
     cudaEventRecord(ctx->ev0, st);
-    cudaError_t e = tiles ? owl_launch_fold(a, ctx->n_sm * per_sm, st) : cudaSuccess;
+    cudaError_t e = items ? owl_launch_fold(a, ctx->n_sm * per_sm, st) : cudaSuccess;
     cudaEventRecord(ctx->ev1, st);
     if (e == cudaSuccess) e = cudaMemcpyAsync(&hs, ctx->d_status, sizeof hs, cudaMemcpyDeviceToHost, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
@@ -293,11 +323,13 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     else {
       float ms = 0;
       cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1);
-      if (tiles) ctx->fold_launches += 1;
+      if (items) ctx->fold_launches += 1;
       ctx->last_fold_ms = ms;
       ctx->last_fold_records = nrec;
       ctx->total_fold_ms += ms;
       ctx->total_fold_records += nrec;
+      if (getenv("OWL_FOLD_VERBOSE")) fprintf(stderr, "[owl] fold: %llu records %.3f ms flushes %llu bypass %llu claims %llu\n",
+        (unsigned long long)nrec, ms, hs.n_flush, hs.n_bypass, hs.n_claim);
     }
   }
   if (status == OWL_OK) {
@@ -455,6 +487,7 @@ OWL_API owl_status owl_ctx_destroy(owl_ctx* ctx) {
   if (!ctx) return OWL_OK;
   cudaSetDevice(ctx->device);
   owl_dev_free(ctx->d_status);
+  owl_dev_trim(ctx->device);
   if (ctx->ev0) cudaEventDestroy(ctx->ev0);
   if (ctx->ev1) cudaEventDestroy(ctx->ev1);
   delete ctx;
@@ -836,7 +869,7 @@ OWL_API owl_status owl_partition_evidence(owl_ctx* ctx, const owl_adcfg* partial
   owl_adcfg* g = const_cast<owl_adcfg*>(partial);
   owl_status s = ensure_sorted(g);
   if (s != OWL_OK) return s;
-  if (g->send) { cudaFree(g->send); g->send = nullptr; }
+  if (g->send) { owl_dev_free(g->send); g->send = nullptr; }
   std::vector<uint64_t> counts(world);
   CUDA_TRY(owl_partition_cells(g->sorted, world, &g->send, counts.data(), ctx->stream), "partition");
   for (int w = 0; w < world; ++w) send_bytes[w] = counts[w] * sizeof(ExchangeCell);

@@ -55,6 +55,9 @@ struct FoldStatus {
   unsigned int overflow;            /* bitmask of tables that exceeded their load limit             */
   unsigned int limit;               /* bitmask: 1 = slot/j field limit exceeded, 2 = visits map full */
   unsigned long long tile_counter;  /* persistent-kernel work counter                               */
+  unsigned long long n_flush;       /* shared-table flushes (all CTAs)                              */
+  unsigned long long n_bypass;      /* address inserts that went straight to the global table      */
+  unsigned long long n_claim;       /* shared-table cells claimed                                   */
 };
 
 /* One segment as the fold kernel sees it */
@@ -69,13 +72,23 @@ struct FoldSeg {
   uint32_t _pad;
 };
 
+/* A work item of the fold is (group, tile position p): warp w of the CTA folds tile p of the group's
+   w-th segment.  Groups hold up to 32 segments of one slot (run batching). */
+struct FoldGroup {
+  uint64_t item0;     /* first work-item id of this group */
+  uint32_t first_seg; /* index of its first member in FoldArgs::segs */
+  uint32_t n_members;
+};
+
 struct FoldArgs {
   const FoldSeg* segs;
-  uint32_t n_segs;
+  const FoldGroup* groups;
+  uint32_t n_groups;
   uint32_t tile_shift;   /* tile = 1 << tile_shift records */
-  uint64_t n_tiles;
+  uint64_t n_items;
   DevTable tab[T_NUM];
   FoldStatus* status;
+  uint32_t mode; /* experiment switch (OWL_FOLD_MODE): 0 normal, 1 no address inserts, 2 stream only */
 };
 
 /* ---- launchers (owl_fold.cu, owl_tables.cu, owl_ks.cu, owl_exchange.cu) ---- */
@@ -134,6 +147,7 @@ cudaError_t owl_absorb_cells(const DevTable* tabs, const ExchangeCell* cells, ui
 /* device memory helpers (owl_tables.cu) */
 void* owl_dev_alloc(size_t bytes);
 void owl_dev_free(void* p);
+void owl_dev_trim(int device); /* return cached blocks to CUDA */
 
 /* host-side key helpers */
 static inline uint64_t owl_mix64(uint64_t x) {

@@ -1,6 +1,6 @@
 /*
- * owl_ks.cu — A6: batched two-sample Kolmogorov-Smirnov tests (Eqs. 1-4), one warp per
- * attribute pair, on the canonical (sorted) tables of E_fix and E_rnd.
+ * owl_ks.cu — A6: batched two-sample Kolmogorov-Smirnov tests (Eqs. 1-4) on the canonical
+ * (sorted) tables of E_fix and E_rnd.
  *
  *   H_cf  per node (Eqs. 5-8): the node's triple cells (prev, next), row-major with S last
  *         (reading R6) — exactly the sorted triple table's order inside one key_hi = (slot, bb).
@@ -9,13 +9,18 @@
  * An attribute is tested only when it is present on both sides of an aligned slot pair (reading R9).
  *
  * Samples are histogram x-values repeated by their counts (R4).  With A_t, B_t the fix / rnd counts at or
- * below t, F_X(t) = A_t/n and F_Y(t) = B_t/m, so D = sup|F_X - F_Y| = K/(n m), K = max_t |A_t m - B_t n|,
- * evaluated exactly in 128-bit integers at every x of either side (each lane: own cell's prefix sum plus a
- * binary search of the other side).  Then, in fp64 with round-to-nearest intrinsics and no FMA, in the
- * fixed order of DESIGN.md §3: D = K/(n*m); w = (n*m)/(n+m); x = (2*(D*D))*w; p = 2*exp(-x);
- * fail = p < significance.
+ * below t, F_X(t) = A_t/n and F_Y(t) = B_t/m, so D = sup|F_X - F_Y| = K/(n m) with the exact 128-bit
+ * K = max_t |A_t m - B_t n|, evaluated at every distinct x of the union of both sides.
+ *
+ * Work decomposition: the sorted union of an attribute pair's two cell lists is cut into units of 1024
+ * union positions; one warp per unit, each lane walks 32 consecutive union positions starting from a
+ * merge-path split (binary search), carrying the segmented prefix sums A and B, and evaluates |A m - B n|
+ * after the last occurrence of each x.  Unit maxima are reduced per pair, then D and p are computed in
+ * fp64 with round-to-nearest intrinsics and no FMA, in the fixed order of DESIGN.md §3:
+ *   D = K/(n*m); w = (n*m)/(n+m); x = (2*(D*D))*w; p = 2*exp(-x); fail = p < significance.
  */
 #include <cub/cub.cuh>
+#include <thrust/iterator/counting_iterator.h>
 #include <cuda_runtime.h>
 
 #include "owl_internal.h"
@@ -23,6 +28,8 @@
 namespace {
 
 typedef unsigned __int128 u128;
+#define UNIT 1024u
+#define PER_LANE (UNIT / 32u)
 
 __global__ void extract_hi_kernel(const Key128* k, uint64_t n, unsigned long long* hi, unsigned char* start) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
@@ -40,7 +47,7 @@ __device__ __forceinline__ unsigned long long with_slot(int tbl, unsigned long l
                        : ((hi & 0xFFFFFFFFull) | ((unsigned long long)s << 32));
 }
 
-/* pairs (attribute index on fix side, attribute index on rnd side) */
+/* pairs (attribute index on the fix side, attribute index on the rnd side) */
 __global__ void pair_kernel(int tbl, const unsigned long long* hif, const uint64_t* stf, uint64_t naf,
                             const unsigned long long* hir, const uint64_t* str, uint64_t nar, const uint32_t* map,
                             uint32_t nmap, uint2* pairs, unsigned long long* npairs) {
@@ -58,6 +65,89 @@ __global__ void pair_kernel(int tbl, const unsigned long long* hif, const uint64
       const unsigned long long o = atomicAdd(npairs, 1ull);
       pairs[o] = make_uint2((uint32_t)i, (uint32_t)lo);
     }
+  }
+}
+
+struct Range {
+  uint64_t fb, fe, rb, re;
+};
+__device__ __forceinline__ Range range_of(const uint2 pr, const uint64_t* stf, uint64_t naf, uint64_t nf,
+                                          const uint64_t* str, uint64_t nar, uint64_t nr) {
+  Range r;
+  r.fb = stf[pr.x];
+  r.fe = pr.x + 1 < naf ? stf[pr.x + 1] : nf;
+  r.rb = str[pr.y];
+  r.re = pr.y + 1 < nar ? str[pr.y + 1] : nr;
+  return r;
+}
+
+__global__ void units_kernel(const uint2* pairs, uint64_t np, const uint64_t* stf, uint64_t naf, uint64_t nf,
+                             const uint64_t* str, uint64_t nar, uint64_t nr, unsigned long long* nunits) {
+  for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < np; p += (uint64_t)gridDim.x * blockDim.x) {
+    const Range r = range_of(pairs[p], stf, naf, nf, str, nar, nr);
+    const uint64_t U = (r.fe - r.fb) + (r.re - r.rb);
+    nunits[p] = (U + UNIT - 1) / UNIT;
+  }
+}
+
+__device__ __forceinline__ u128 absdiff(u128 a, u128 b) { return a > b ? a - b : b - a; }
+
+/* one warp per unit: partial K of union positions [u*UNIT, (u+1)*UNIT) of one pair */
+__global__ void ks_unit_kernel(const Key128* fk, const unsigned long long* fpre, uint64_t nf, const uint64_t* stf,
+                               uint64_t naf, const Key128* rk, const unsigned long long* rpre, uint64_t nr,
+                               const uint64_t* str, uint64_t nar, const uint2* pairs, uint64_t np,
+                               const unsigned long long* uoff, uint64_t total_units, u128* partial) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp0 = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t u = warp0; u < total_units; u += nwarps) {
+    uint64_t lo = 0, hi = np; /* pair of unit u: last p with uoff[p] <= u */
+    while (hi - lo > 1) {
+      const uint64_t mid = (lo + hi) >> 1;
+      if (uoff[mid] <= u) lo = mid; else hi = mid;
+    }
+    const Range r = range_of(pairs[lo], stf, naf, nf, str, nar, nr);
+    const uint64_t nfa = r.fe - r.fb, nra = r.re - r.rb;
+    const unsigned long long n = fpre[r.fe - 1], m = rpre[r.re - 1];
+    const uint64_t d0 = (u - uoff[lo]) * UNIT + (uint64_t)lane * PER_LANE;
+    const uint64_t d1 = d0 + PER_LANE < nfa + nra ? d0 + PER_LANE : nfa + nra;
+    u128 K = 0;
+    if (d0 < d1) {
+      /* merge-path split: i fix elements among the first d0 union positions (ties: fix first) */
+      uint64_t a = d0 > nra ? d0 - nra : 0, b = d0 < nfa ? d0 : nfa;
+      while (a < b) {
+        const uint64_t mid = (a + b) >> 1;
+        if (fk[r.fb + mid].lo <= rk[r.rb + (d0 - mid - 1)].lo) a = mid + 1; else b = mid;
+      }
+      uint64_t i = a, j = d0 - a;
+      unsigned long long A = i ? fpre[r.fb + i - 1] : 0ull, B = j ? rpre[r.rb + j - 1] : 0ull;
+      for (uint64_t d = d0; d < d1; ++d) {
+        unsigned long long x;
+        if (i < nfa && (j >= nra || fk[r.fb + i].lo <= rk[r.rb + j].lo)) {
+          x = fk[r.fb + i].lo;
+          A = fpre[r.fb + i];
+          ++i;
+        } else {
+          x = rk[r.rb + j].lo;
+          B = rpre[r.rb + j];
+          ++j;
+        }
+        /* evaluate after the last occurrence of x in the union */
+        const bool more_f = i < nfa && fk[r.fb + i].lo == x;
+        const bool more_r = j < nra && rk[r.rb + j].lo == x;
+        if (!more_f && !more_r) {
+          const u128 dd = absdiff((u128)A * m, (u128)B * n);
+          if (dd > K) K = dd;
+        }
+      }
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+      const unsigned long long khi = __shfl_xor_sync(0xFFFFFFFFu, (unsigned long long)(K >> 64), o);
+      const unsigned long long klo = __shfl_xor_sync(0xFFFFFFFFu, (unsigned long long)K, o);
+      const u128 other = ((u128)khi << 64) | klo;
+      if (other > K) K = other;
+    }
+    if (lane == 0) partial[u] = K;
   }
 }
 
@@ -79,68 +169,35 @@ __device__ double u128_to_double_rn(u128 v) {
   return scalbn((double)mant, e);
 }
 
-__device__ __forceinline__ u128 absdiff(u128 a, u128 b) { return a > b ? a - b : b - a; }
-
-__global__ void ks_kernel(const Key128* fk, const unsigned long long* fpre, uint64_t nf, const uint64_t* stf, uint64_t naf,
-                          const Key128* rk, const unsigned long long* rpre, uint64_t nr, const uint64_t* str, uint64_t nar,
-                          const uint2* pairs, uint64_t npairs, double significance, KsOutRow* out) {
-  const int lane = threadIdx.x & 31;
-  const uint64_t warp0 = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
-  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-  for (uint64_t w = warp0; w < npairs; w += nwarps) {
-    const uint2 pr = pairs[w];
-    const uint64_t fb = stf[pr.x], fe = pr.x + 1 < naf ? stf[pr.x + 1] : nf;
-    const uint64_t rb = str[pr.y], re = pr.y + 1 < nar ? str[pr.y + 1] : nr;
-    const unsigned long long n = fpre[fe - 1], m = rpre[re - 1];
+__global__ void ks_final_kernel(const Key128* fk, const unsigned long long* fpre, uint64_t nf, const uint64_t* stf,
+                                uint64_t naf, const Key128* rk, const unsigned long long* rpre, uint64_t nr,
+                                const uint64_t* str, uint64_t nar, const uint2* pairs, uint64_t np,
+                                const unsigned long long* uoff, const unsigned long long* nunits, const u128* partial,
+                                double significance, KsOutRow* out) {
+  for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < np; p += (uint64_t)gridDim.x * blockDim.x) {
+    const Range r = range_of(pairs[p], stf, naf, nf, str, nar, nr);
+    const unsigned long long n = fpre[r.fe - 1], m = rpre[r.re - 1];
     u128 K = 0;
-    for (uint64_t i = fb + lane; i < fe; i += 32) {
-      const unsigned long long x = fk[i].lo;
-      uint64_t lo = rb, hi = re; /* first rnd cell with lo > x */
-      while (lo < hi) {
-        const uint64_t mid = (lo + hi) >> 1;
-        if (rk[mid].lo <= x) lo = mid + 1; else hi = mid;
-      }
-      const unsigned long long B = lo > rb ? rpre[lo - 1] : 0ull;
-      const u128 d = absdiff((u128)fpre[i] * m, (u128)B * n);
-      if (d > K) K = d;
-    }
-    for (uint64_t i = rb + lane; i < re; i += 32) {
-      const unsigned long long x = rk[i].lo;
-      uint64_t lo = fb, hi = fe;
-      while (lo < hi) {
-        const uint64_t mid = (lo + hi) >> 1;
-        if (fk[mid].lo <= x) lo = mid + 1; else hi = mid;
-      }
-      const unsigned long long A = lo > fb ? fpre[lo - 1] : 0ull;
-      const u128 d = absdiff((u128)A * m, (u128)rpre[i] * n);
-      if (d > K) K = d;
-    }
-    for (int o = 16; o > 0; o >>= 1) {
-      const unsigned long long khi = __shfl_xor_sync(0xFFFFFFFFu, (unsigned long long)(K >> 64), o);
-      const unsigned long long klo = __shfl_xor_sync(0xFFFFFFFFu, (unsigned long long)K, o);
-      const u128 other = ((u128)khi << 64) | klo;
-      if (other > K) K = other;
-    }
-    if (lane == 0) {
-      const double nd = __ull2double_rn(n), md = __ull2double_rn(m);
-      const double nm = __dmul_rn(nd, md);
-      const double D = __ddiv_rn(u128_to_double_rn(K), nm);
-      const double wgt = __ddiv_rn(nm, __dadd_rn(nd, md));
-      const double x = __dmul_rn(__dmul_rn(2.0, __dmul_rn(D, D)), wgt);
-      const double p = __dmul_rn(2.0, exp(-x));
-      KsOutRow r;
-      r.hi_f = fk[fb].hi;
-      r.hi_r = rk[rb].hi;
-      r.n = n;
-      r.m = m;
-      r.K_lo = (unsigned long long)K;
-      r.K_hi = (unsigned long long)(K >> 64);
-      r.D = D;
-      r.p = p;
-      r.fail = p < significance ? 1u : 0u;
-      r._pad = 0;
-      out[w] = r;
-    }
+    for (unsigned long long q = 0; q < nunits[p]; ++q)
+      if (partial[uoff[p] + q] > K) K = partial[uoff[p] + q];
+    const double nd = __ull2double_rn(n), md = __ull2double_rn(m);
+    const double nm = __dmul_rn(nd, md);
+    const double D = __ddiv_rn(u128_to_double_rn(K), nm);
+    const double wgt = __ddiv_rn(nm, __dadd_rn(nd, md));
+    const double x = __dmul_rn(__dmul_rn(2.0, __dmul_rn(D, D)), wgt);
+    const double pv = __dmul_rn(2.0, exp(-x));
+    KsOutRow o;
+    o.hi_f = fk[r.fb].hi;
+    o.hi_r = rk[r.rb].hi;
+    o.n = n;
+    o.m = m;
+    o.K_lo = (unsigned long long)K;
+    o.K_hi = (unsigned long long)(K >> 64);
+    o.D = D;
+    o.p = pv;
+    o.fail = pv < significance ? 1u : 0u;
+    o._pad = 0;
+    out[p] = o;
   }
 }
 
@@ -152,7 +209,7 @@ struct Side {
   unsigned long long* nattr = nullptr;
   uint64_t na = 0;
   void free_all() {
-    cudaFree(hi); cudaFree(st); cudaFree(pre); cudaFree(starts); cudaFree(nattr);
+    owl_dev_free(hi); owl_dev_free(st); owl_dev_free(pre); owl_dev_free(starts); owl_dev_free(nattr);
   }
 };
 
@@ -164,23 +221,26 @@ int grid_for(uint64_t n, int block) {
 
 cudaError_t prepare(const SortedTable& t, Side& s, cudaStream_t st) {
   const uint64_t n = t.n;
-  if (cudaMalloc(&s.hi, (n + 1) * 8) || cudaMalloc(&s.st, n + 1) || cudaMalloc(&s.pre, (n + 1) * 8) ||
-      cudaMalloc(&s.starts, (n + 1) * 8) || cudaMalloc(&s.nattr, 8))
-    return cudaErrorMemoryAllocation;
+  s.hi = (unsigned long long*)owl_dev_alloc((n + 1) * 8);
+  s.st = (unsigned char*)owl_dev_alloc(n + 1);
+  s.pre = (unsigned long long*)owl_dev_alloc((n + 1) * 8);
+  s.starts = (uint64_t*)owl_dev_alloc((n + 1) * 8);
+  s.nattr = (unsigned long long*)owl_dev_alloc(8);
+  if (!s.hi || !s.st || !s.pre || !s.starts || !s.nattr) return cudaErrorMemoryAllocation;
   if (!n) return cudaSuccess;
   extract_hi_kernel<<<grid_for(n, 256), 256, 0, st>>>(t.k, n, s.hi, s.st);
   size_t t1 = 0, t2 = 0;
-  cub::DeviceSelect::Flagged(nullptr, t1, cub::CountingInputIterator<uint64_t>(0), s.st, s.starts, s.nattr, (int64_t)n, st);
+  cub::DeviceSelect::Flagged(nullptr, t1, thrust::counting_iterator<uint64_t>(0), s.st, s.starts, s.nattr, (int64_t)n, st);
   cub::DeviceScan::InclusiveSumByKey(nullptr, t2, s.hi, t.c, s.pre, (int64_t)n, cub::Equality(), st);
-  void* tmp = nullptr;
-  if (cudaMalloc(&tmp, (t1 > t2 ? t1 : t2) + 16)) return cudaErrorMemoryAllocation;
-  cudaError_t e = cub::DeviceSelect::Flagged(tmp, t1, cub::CountingInputIterator<uint64_t>(0), s.st, s.starts, s.nattr,
+  void* tmp = owl_dev_alloc((t1 > t2 ? t1 : t2) + 16);
+  if (!tmp) return cudaErrorMemoryAllocation;
+  cudaError_t e = cub::DeviceSelect::Flagged(tmp, t1, thrust::counting_iterator<uint64_t>(0), s.st, s.starts, s.nattr,
                                              (int64_t)n, st);
   if (e == cudaSuccess) e = cub::DeviceScan::InclusiveSumByKey(tmp, t2, s.hi, t.c, s.pre, (int64_t)n, cub::Equality(), st);
   unsigned long long na = 0;
   if (e == cudaSuccess) e = cudaMemcpyAsync(&na, s.nattr, 8, cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  cudaFree(tmp);
+  owl_dev_free(tmp);
   s.na = na;
   return e;
 }
@@ -194,14 +254,19 @@ cudaError_t owl_ks_run(int tbl, const SortedTable& f, const SortedTable& r, cons
   Side sf, sr;
   uint32_t* dmap = nullptr;
   uint2* pairs = nullptr;
-  unsigned long long* npairs = nullptr;
+  unsigned long long *npairs = nullptr, *nunits = nullptr, *uoff = nullptr;
+  u128* partial = nullptr;
   KsOutRow* dout = nullptr;
+  void* tmp = nullptr;
   cudaError_t e = prepare(f, sf, st);
   if (e == cudaSuccess) e = prepare(r, sr, st);
   unsigned long long np = 0;
-  if (e == cudaSuccess && cudaMalloc(&dmap, slot_f2r.size() * 4)) e = cudaErrorMemoryAllocation;
-  if (e == cudaSuccess && (cudaMalloc(&pairs, (sf.na + 1) * sizeof(uint2)) || cudaMalloc(&npairs, 8)))
-    e = cudaErrorMemoryAllocation;
+  if (e == cudaSuccess) {
+    dmap = (uint32_t*)owl_dev_alloc(slot_f2r.size() * 4);
+    pairs = (uint2*)owl_dev_alloc((sf.na + 1) * sizeof(uint2));
+    npairs = (unsigned long long*)owl_dev_alloc(8);
+    if (!dmap || !pairs || !npairs) e = cudaErrorMemoryAllocation;
+  }
   if (e == cudaSuccess) {
     cudaMemcpyAsync(dmap, slot_f2r.data(), slot_f2r.size() * 4, cudaMemcpyHostToDevice, st);
     cudaMemsetAsync(npairs, 0, 8, st);
@@ -211,10 +276,33 @@ cudaError_t owl_ks_run(int tbl, const SortedTable& f, const SortedTable& r, cons
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   }
   if (e == cudaSuccess && np) {
-    if (cudaMalloc(&dout, np * sizeof(KsOutRow))) e = cudaErrorMemoryAllocation;
+    nunits = (unsigned long long*)owl_dev_alloc(np * 8);
+    uoff = (unsigned long long*)owl_dev_alloc((np + 1) * 8);
+    dout = (KsOutRow*)owl_dev_alloc(np * sizeof(KsOutRow));
+    if (!nunits || !uoff || !dout) e = cudaErrorMemoryAllocation;
+    unsigned long long total = 0;
     if (e == cudaSuccess) {
-      ks_kernel<<<grid_for(np * 32, 256), 256, 0, st>>>(f.k, sf.pre, f.n, sf.starts, sf.na, r.k, sr.pre, r.n, sr.starts,
-                                                        sr.na, pairs, np, significance, dout);
+      units_kernel<<<grid_for(np, 256), 256, 0, st>>>(pairs, np, sf.starts, sf.na, f.n, sr.starts, sr.na, r.n, nunits);
+      size_t tb = 0;
+      cub::DeviceScan::InclusiveSum(nullptr, tb, nunits, uoff + 1, (int64_t)np, st);
+      tmp = owl_dev_alloc(tb + 16);
+      if (!tmp) e = cudaErrorMemoryAllocation;
+      if (e == cudaSuccess) {
+        cudaMemsetAsync(uoff, 0, 8, st);
+        e = cub::DeviceScan::InclusiveSum(tmp, tb, nunits, uoff + 1, (int64_t)np, st);
+      }
+      if (e == cudaSuccess) e = cudaMemcpyAsync(&total, uoff + np, 8, cudaMemcpyDeviceToHost, st);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    }
+    if (e == cudaSuccess) {
+      partial = (u128*)owl_dev_alloc((total + 1) * sizeof(u128));
+      if (!partial) e = cudaErrorMemoryAllocation;
+    }
+    if (e == cudaSuccess) {
+      ks_unit_kernel<<<grid_for(total * 32, 256), 256, 0, st>>>(f.k, sf.pre, f.n, sf.starts, sf.na, r.k, sr.pre, r.n,
+                                                                  sr.starts, sr.na, pairs, np, uoff, total, partial);
+      ks_final_kernel<<<grid_for(np, 128), 128, 0, st>>>(f.k, sf.pre, f.n, sf.starts, sf.na, r.k, sr.pre, r.n, sr.starts,
+                                                         sr.na, pairs, np, uoff, nunits, partial, significance, dout);
       rows.resize(np);
       e = cudaMemcpyAsync(rows.data(), dout, np * sizeof(KsOutRow), cudaMemcpyDeviceToHost, st);
       if (e == cudaSuccess) e = cudaStreamSynchronize(st);
@@ -222,7 +310,8 @@ cudaError_t owl_ks_run(int tbl, const SortedTable& f, const SortedTable& r, cons
   }
   sf.free_all();
   sr.free_all();
-  cudaFree(dmap); cudaFree(pairs); cudaFree(npairs); cudaFree(dout);
+  owl_dev_free(dmap); owl_dev_free(pairs); owl_dev_free(npairs); owl_dev_free(nunits); owl_dev_free(uoff);
+  owl_dev_free(dout); owl_dev_free(partial); owl_dev_free(tmp);
   if (e == cudaSuccess) e = cudaGetLastError();
   return e;
 }

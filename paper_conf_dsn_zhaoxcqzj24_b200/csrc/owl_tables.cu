@@ -4,8 +4,13 @@
  * P:L227-229), and stable bucketing of channel-order input by warp (reading R17).
  */
 #include <cub/cub.cuh>
+#include <thrust/iterator/counting_iterator.h>
 #include <cuda/std/tuple>
 #include <cuda_runtime.h>
+
+#include <map>
+#include <mutex>
+#include <vector>
 
 #include "owl_device.cuh"
 #include "owl_internal.h"
@@ -124,13 +129,59 @@ int grid_for(uint64_t n, int block) {
 
 }  // namespace
 
+/* Caching device allocator: blocks are rounded up to a power of two (>= 256 B) and recycled per device,
+   so the per-call scratch of build / sort / diff / KS never hits cudaMalloc / cudaFree (which synchronize
+   the device) in steady state.  All library work of a context runs on its one stream, so a block freed
+   by one call and reused by the next is ordered by that stream. */
+namespace {
+std::mutex g_pool_mu;
+std::map<std::pair<int, size_t>, std::vector<void*>> g_pool;   /* (device, size) -> free blocks */
+std::map<void*, std::pair<int, size_t>> g_live;                /* block -> (device, size) */
+}  // namespace
+
 void* owl_dev_alloc(size_t bytes) {
+  size_t sz = 256;
+  while (sz < bytes) sz <<= 1;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  auto it = g_pool.find({dev, sz});
   void* p = nullptr;
-  if (cudaMalloc(&p, bytes ? bytes : 16) != cudaSuccess) return nullptr;
+  if (it != g_pool.end() && !it->second.empty()) {
+    p = it->second.back();
+    it->second.pop_back();
+  } else if (cudaMalloc(&p, sz) != cudaSuccess) {
+    cudaGetLastError();
+    for (auto& f : g_pool) /* release cached blocks of this device and retry once */
+      if (f.first.first == dev) {
+        for (void* q : f.second) cudaFree(q);
+        f.second.clear();
+      }
+    if (cudaMalloc(&p, sz) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+  }
+  g_live[p] = {dev, sz};
   return p;
 }
+
 void owl_dev_free(void* p) {
-  if (p) cudaFree(p);
+  if (!p) return;
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  auto it = g_live.find(p);
+  if (it == g_live.end()) return;
+  g_pool[it->second].push_back(p);
+  g_live.erase(it);
+}
+
+void owl_dev_trim(int dev) {
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  for (auto& f : g_pool)
+    if (f.first.first == dev) {
+      for (void* q : f.second) cudaFree(q);
+      f.second.clear();
+    }
 }
 
 cudaError_t owl_table_alloc(DevTable* t, uint64_t cap, cudaStream_t st) {
@@ -213,8 +264,8 @@ cudaError_t owl_diff_sorted(const SortedTable& a, const SortedTable& b, std::vec
   if (e == cudaSuccess) {
     diff_flag_kernel<<<grid_for(na > nb ? na : nb, 256), 256, 0, st>>>(a.k, a.c, na, b.k, b.c, nb, fa, cboa, fb);
     size_t tmp = 0, tmp2 = 0;
-    cub::DeviceSelect::Flagged(nullptr, tmp, cub::CountingInputIterator<uint64_t>(0), fa, ia, nsel, (int64_t)na, st);
-    cub::DeviceSelect::Flagged(nullptr, tmp2, cub::CountingInputIterator<uint64_t>(0), fb, ib, nsel + 1, (int64_t)nb, st);
+    cub::DeviceSelect::Flagged(nullptr, tmp, thrust::counting_iterator<uint64_t>(0), fa, ia, nsel, (int64_t)na, st);
+    cub::DeviceSelect::Flagged(nullptr, tmp2, thrust::counting_iterator<uint64_t>(0), fb, ib, nsel + 1, (int64_t)nb, st);
     if (tmp2 > tmp) tmp = tmp2;
     dt = owl_dev_alloc(tmp);
     if (!dt) e = cudaErrorMemoryAllocation;
@@ -222,12 +273,12 @@ cudaError_t owl_diff_sorted(const SortedTable& a, const SortedTable& b, std::vec
   unsigned long long hn[2] = {0, 0};
   if (e == cudaSuccess) {
     size_t tmp = 0;
-    cub::DeviceSelect::Flagged(nullptr, tmp, cub::CountingInputIterator<uint64_t>(0), fa, ia, nsel, (int64_t)na, st);
-    e = cub::DeviceSelect::Flagged(dt, tmp, cub::CountingInputIterator<uint64_t>(0), fa, ia, nsel, (int64_t)na, st);
+    cub::DeviceSelect::Flagged(nullptr, tmp, thrust::counting_iterator<uint64_t>(0), fa, ia, nsel, (int64_t)na, st);
+    e = cub::DeviceSelect::Flagged(dt, tmp, thrust::counting_iterator<uint64_t>(0), fa, ia, nsel, (int64_t)na, st);
     tmp = 0;
-    cub::DeviceSelect::Flagged(nullptr, tmp, cub::CountingInputIterator<uint64_t>(0), fb, ib, nsel + 1, (int64_t)nb, st);
+    cub::DeviceSelect::Flagged(nullptr, tmp, thrust::counting_iterator<uint64_t>(0), fb, ib, nsel + 1, (int64_t)nb, st);
     if (e == cudaSuccess)
-      e = cub::DeviceSelect::Flagged(dt, tmp, cub::CountingInputIterator<uint64_t>(0), fb, ib, nsel + 1, (int64_t)nb, st);
+      e = cub::DeviceSelect::Flagged(dt, tmp, thrust::counting_iterator<uint64_t>(0), fb, ib, nsel + 1, (int64_t)nb, st);
     if (e == cudaSuccess) {
       gather_diff_kernel<<<grid_for(na, 256), 256, 0, st>>>(ia, nsel, a.k, a.c, cboa, 1, da);
       gather_diff_kernel<<<grid_for(nb, 256), 256, 0, st>>>(ib, nsel + 1, b.k, b.c, nullptr, 0, db);

@@ -251,3 +251,20 @@ def test_full_size_c2_run_parity(ctx):
         assert int(ev["addr"]["count"].sum()) + int(ev["node"]["count"].sum()) == n_rec
     finally:
         ctx.forget_runs([0, 1, 2, 3])
+
+
+def test_work_queue_stress_long_warps(ctx):
+    """C3 traced warps (~107K records) span many tiles, so most tiles hold no warp start and warps re-pop the
+    CTA queue immediately; 40 identical FIX runs must give exactly 40 x one run (a duplicated or skipped
+    tile would break it), and one run must match the oracle."""
+    p = tracegen.Params.preset(3, grid_div=16, runs_fix=40, runs_rnd=0)
+    runs = list(range(40))
+    ctx.ingest(_gpu_segments(p, runs))
+    try:
+        one = ctx.build([0])
+        assert one.export() == oracle.build(_oracle_segments(p, [0])[0]).export()
+        ev, o = H.parse_blob(ctx.build(runs).export()), H.parse_blob(one.export())
+        for t in ("node", "edge", "triple", "addr"):
+            assert np.array_equal(ev[t]["count"], 40 * o[t]["count"]), t
+    finally:
+        ctx.forget_runs(runs)
