@@ -151,6 +151,78 @@ def run_reference(args):
     }), flush=True)
 
 
+def count_launches(step):
+    """Kernels launched by one (untimed) step, from a CUDA-activity trace: (ours, names).  'Ours' = every
+    kernel compiled into libowl.so (fold / tables / KS / exchange kernels and the CUB sort kernels
+    instantiated there); torch's own memset/copy activity is not a kernel and is not counted."""
+    import torch
+    from torch.profiler import ProfilerActivity, profile
+    with profile(activities=[ProfilerActivity.CUDA]) as prof:
+        step()
+        torch.cuda.synchronize()
+    names = {}
+    for ev in prof.events():
+        if getattr(ev, "device_type", None) is not None and str(ev.device_type).endswith("CUDA"):
+            n = ev.name
+            if n.lower().startswith(("memcpy", "memset")):
+                continue
+            names[n] = names.get(n, 0) + 1
+    return sum(names.values()), names
+
+
+def e2e_leg(args, p, api, tracegen, dev, stream, n_runs_e2e):
+    """Same metric through the public C ABI with HOST records: every step stages the runs' records from
+    pinned host memory into HBM inside owl_build_adcfg (OWL_SEG_HOST_RECORDS), folds, diffs and runs the
+    leak test, whose rows come back to the host (D2H).  A subset of the workload's runs (stated) keeps the
+    pinned host footprint bounded."""
+    import torch
+    ctx = api.Context(dev.index)
+    base_run = 1 << 20  # run ids disjoint from the device-resident leg
+    runs_f = [r for r in range(p.n_runs) if tracegen.run_class(p, r) == 0][: n_runs_e2e // 2]
+    runs_r = [r for r in range(p.n_runs) if tracegen.run_class(p, r) == 1][: n_runs_e2e // 2]
+    segs, hold, n_rec = [], [], 0
+    for r in runs_f + runs_r:
+        for m in tracegen.run_segments(p, r):
+            buf, n = tracegen.device_records(p, r, m.seq, device=dev, stream=stream)
+            h = torch.empty(buf.shape, dtype=buf.dtype, pin_memory=True)
+            h.copy_(buf)
+            del buf
+            hold.append(h)
+            segs.append(api.Segment(base_run + r, m.input_class, m.seq, m.n_warps, m.kernel_id, h, n,
+                                    flags=api.OWL_SEG_WARP_MAJOR | api.OWL_SEG_HOST_RECORDS))
+            n_rec += n
+    torch.cuda.synchronize()
+    ctx.ingest(segs, stream)
+    rf = [base_run + r for r in runs_f]
+    rr = [base_run + r for r in runs_r]
+    d2h = [0]
+
+    def step():
+        ef, er = ctx.build(rf), ctx.build(rr)
+        d = ctx.diff(ef, er)
+        lk = ctx.leak_test(ef, er, 0.05)
+        d2h[0] = d.nbytes + lk.nbytes
+        ef.destroy()
+        er.destroy()
+
+    for _ in range(max(1, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    steps = max(1, min(args.steps, 3))
+    e0.record(stream)
+    for _ in range(steps):
+        step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    del ctx, segs, hold
+    return {"value": n_rec / (ms / 1e3), "unit": "records/s", "h2d_bytes_per_step": 16 * n_rec,
+            "d2h_bytes_per_step": d2h[0], "ms_per_step": ms, "records_per_step": n_rec,
+            "sample": f"{len(rf)} FIX + {len(rr)} RND runs of the same workload from pinned host memory, "
+                      f"{steps} steps"}
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -253,12 +325,19 @@ def run_ours(args):
                      "note": f"16 B/record algorithmic; {st['fold_launches']} fold launches, "
                              f"{fold_ms:.2f} ms avg (CUDA events on the launch stream); peak {peak_src}"},
         "clocks": ck,
-        "gpu_launches": None,
         "fold_share_of_step": (st["total_fold_ms"] / args.steps) / ms,
         "breakdown_ms": {k: v / args.steps for k, v in brk.items()} if args.breakdown else None,
         "result": {"n_diff_rows": out.get("n_diff"), "n_leaks": out.get("n_leaks"),
                    "cells_fix": out.get("info_f", {}).get("n_cells"), "cells_rnd": out.get("info_r", {}).get("n_cells")},
     }
+    n_launch, names = count_launches(step)
+    res["gpu_launches"] = n_launch * args.steps
+    res["gpu_launches_per_step"] = names
+    if not args.no_e2e:
+        del segs
+        ctx.forget_runs(my_runs)
+        torch.cuda.empty_cache()
+        res["e2e"] = e2e_leg(args, p, api, tracegen, dev, stream, args.e2e_runs)
     if rank == 0 and not args.no_cpu:
         res["cpu_baseline"] = cpu_baseline(cfg, args.cpu_seconds)
     if rank == 0:
@@ -276,6 +355,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--runs", type=int, default=0, help="limit runs per GPU (debug)")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-runs", type=int, default=20, help="runs (half FIX, half RND) in the host-records e2e leg")
     ap.add_argument("--breakdown", action="store_true", help="host-timed per-call breakdown (syncs between calls)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     args = ap.parse_args()

@@ -17,6 +17,17 @@ __device__ __forceinline__ uint64_t hmix(uint64_t hi, uint64_t lo) {
   return x;
 }
 
+/* Global-table index of a key: multiplicative hash, top log2(cap) bits.  One definition for every
+   kernel that probes a DevTable (fold, merge, absorb), so all agree on a key's home cell. */
+__device__ __forceinline__ uint64_t tab_hash(uint64_t hi, uint64_t lo) {
+  uint64_t x = lo ^ (hi * 0x9E3779B97F4A7C15ull);
+  x ^= x >> 32;
+  return x * 0xD6E8FEB86659FD93ull;
+}
+__device__ __forceinline__ uint32_t tab_shift(uint64_t cap) { /* cap: power of two >= 2 */
+  return (uint32_t)(65 - __ffsll((long long)cap));
+}
+
 __device__ __forceinline__ ulonglong2 cas128_global(unsigned long long* p, unsigned long long cmp_hi,
                                                     unsigned long long cmp_lo, unsigned long long new_hi,
                                                     unsigned long long new_lo) {
@@ -58,7 +69,7 @@ __device__ __forceinline__ ulonglong2 ld_key(const owl_cell* c) {
 /* Insert-or-add into a global table.  Returns false (and flags overflow) if no cell was found. */
 static __device__ __noinline__ bool g_insert(const DevTable& t, int tbl, uint64_t hi, uint64_t lo, uint64_t c, FoldStatus* st) {
   const uint64_t mask = t.cap - 1;
-  uint64_t h = hmix(hi, lo) & mask;
+  uint64_t h = tab_hash(hi, lo) >> tab_shift(t.cap);
   for (uint64_t probe = 0; probe < t.cap; ++probe) {
     owl_cell* cell = t.cells + h;
     ulonglong2 k = ld_key(cell);

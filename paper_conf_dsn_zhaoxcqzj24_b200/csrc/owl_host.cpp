@@ -261,7 +261,9 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     tiles += (s.n_records + (1ull << tile_shift) - 1) >> tile_shift;
     nrec += s.n_records;
   }
-  /* run batching (owl_fold.cu): groups of up to 32 segments of one slot, ascending run */
+  /* run batching (owl_fold.cu): groups of up to owl_fold_runs_per_warp() segments of one slot, ascending run;
+     one warp walks all members of a group at the same tile position */
+  const size_t group_max = (size_t)owl_fold_runs_per_warp();
   std::vector<uint32_t> order(fs.size());
   for (size_t i = 0; i < order.size(); ++i) order[i] = (uint32_t)i;
   std::stable_sort(order.begin(), order.end(), [&](uint32_t x, uint32_t y) { return fs[x].slot < fs[y].slot; });
@@ -271,7 +273,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
   for (size_t i = 0; i < order.size();) {
     size_t e = i;
     uint64_t npos = 0;
-    while (e < order.size() && e - i < 32 && fs[order[e]].slot == fs[order[i]].slot) {
+    while (e < order.size() && e - i < group_max && fs[order[e]].slot == fs[order[i]].slot) {
       npos = std::max<uint64_t>(npos, (fs[order[e]].n + (1ull << tile_shift) - 1) >> tile_shift);
       ++e;
     }

@@ -72,8 +72,8 @@ struct FoldSeg {
   uint32_t _pad;
 };
 
-/* A work item of the fold is (group, tile position p): warp w of the CTA folds tile p of the group's
-   w-th segment.  Groups hold up to 32 segments of one slot (run batching). */
+/* A work item of the fold is (group, tile position p): one warp folds tile p of every segment of the group
+   at once.  Groups hold up to owl_fold_runs_per_warp() segments of one slot (run batching). */
 struct FoldGroup {
   uint64_t item0;     /* first work-item id of this group */
   uint32_t first_seg; /* index of its first member in FoldArgs::segs */
@@ -94,6 +94,7 @@ struct FoldArgs {
 /* ---- launchers (owl_fold.cu, owl_tables.cu, owl_ks.cu, owl_exchange.cu) ---- */
 cudaError_t owl_launch_fold(const FoldArgs& a, int grid, cudaStream_t st);
 int owl_fold_ctas_per_sm();
+int owl_fold_runs_per_warp();
 
 struct Key128 {
   unsigned long long hi, lo;
