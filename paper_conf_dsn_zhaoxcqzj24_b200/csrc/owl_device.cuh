@@ -17,15 +17,15 @@ __device__ __forceinline__ uint64_t hmix(uint64_t hi, uint64_t lo) {
   return x;
 }
 
-/* Global-table index of a key: multiplicative hash, top log2(cap) bits.  One definition for every
-   kernel that probes a DevTable (fold, merge, absorb), so all agree on a key's home cell. */
-__device__ __forceinline__ uint64_t tab_hash(uint64_t hi, uint64_t lo) {
-  uint64_t x = lo ^ (hi * 0x9E3779B97F4A7C15ull);
-  x ^= x >> 32;
-  return x * 0xD6E8FEB86659FD93ull;
-}
-__device__ __forceinline__ uint32_t tab_shift(uint64_t cap) { /* cap: power of two >= 2 */
-  return (uint32_t)(65 - __ffsll((long long)cap));
+/* Global-table home cell of a key: xor of four 32-bit multiplicative hashes of the key words, top
+   log2(cap) bits, rounded down to slot 0 of its bucket; probing is linear over cells from there.  One
+   definition for every kernel that probes a DevTable (fold, merge, absorb), so all agree.
+   cap: power of two, 2 <= cap <= 2^31. */
+__device__ __forceinline__ uint32_t tab_shift(uint64_t cap) { return (uint32_t)(33 - __ffsll((long long)cap)); }
+__device__ __forceinline__ uint32_t tab_index(uint64_t hi, uint64_t lo, uint32_t shift) {
+  const uint32_t h = ((uint32_t)lo * 0x9E3779B1u) ^ ((uint32_t)(lo >> 32) * 0x85EBCA77u) ^
+                     ((uint32_t)hi * 0xC2B2AE3Du) ^ ((uint32_t)(hi >> 32) * 0x27D4EB2Fu);
+  return (h >> shift) & ~1u;
 }
 
 __device__ __forceinline__ ulonglong2 cas128_global(unsigned long long* p, unsigned long long cmp_hi,
@@ -60,7 +60,10 @@ __device__ __forceinline__ ulonglong2 cas128_shared(ulonglong2* p, unsigned long
   return o;
 }
 
-__device__ __forceinline__ ulonglong2 ld_key(const owl_cell* c) {
+__device__ __forceinline__ unsigned long long* cell_key(const DevTable& t, uint64_t i) { return &t.b[i >> 1].key[i & 1][0]; }
+__device__ __forceinline__ unsigned long long* cell_count(const DevTable& t, uint64_t i) { return &t.b[i >> 1].count[i & 1]; }
+
+__device__ __forceinline__ ulonglong2 ld_key(const unsigned long long* c) {
   ulonglong2 k;
   asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(k.x), "=l"(k.y) : "l"(c) : "memory");
   return k;
@@ -69,24 +72,24 @@ __device__ __forceinline__ ulonglong2 ld_key(const owl_cell* c) {
 /* Insert-or-add into a global table.  Returns false (and flags overflow) if no cell was found. */
 static __device__ __noinline__ bool g_insert(const DevTable& t, int tbl, uint64_t hi, uint64_t lo, uint64_t c, FoldStatus* st) {
   const uint64_t mask = t.cap - 1;
-  uint64_t h = tab_hash(hi, lo) >> tab_shift(t.cap);
+  uint64_t h = tab_index(hi, lo, tab_shift(t.cap));
   for (uint64_t probe = 0; probe < t.cap; ++probe) {
-    owl_cell* cell = t.cells + h;
-    ulonglong2 k = ld_key(cell);
+    unsigned long long* key = cell_key(t, h);
+    ulonglong2 k = ld_key(key);
     if (k.x == hi && k.y == lo) {
-      atomicAdd(&cell->count, (unsigned long long)c);
+      atomicAdd(cell_count(t, h), (unsigned long long)c);
       return true;
     }
     if (k.x == OWL_EMPTY_KEY || k.x == hi) { /* empty, being claimed, or a possibly torn read: resolve */
-      ulonglong2 o = cas128_global(&cell->hi, OWL_EMPTY_KEY, OWL_EMPTY_KEY, hi, lo);
+      ulonglong2 o = cas128_global(key, OWL_EMPTY_KEY, OWL_EMPTY_KEY, hi, lo);
       if (o.x == OWL_EMPTY_KEY && o.y == OWL_EMPTY_KEY) {
         unsigned long long f = atomicAdd(t.fill, 1ull);
         if (f + 1 > (t.cap >> 1) + (t.cap >> 2)) atomicOr(&st->overflow, 1u << tbl);
-        atomicAdd(&cell->count, (unsigned long long)c);
+        atomicAdd(cell_count(t, h), (unsigned long long)c);
         return true;
       }
       if (o.x == hi && o.y == lo) {
-        atomicAdd(&cell->count, (unsigned long long)c);
+        atomicAdd(cell_count(t, h), (unsigned long long)c);
         return true;
       }
     }

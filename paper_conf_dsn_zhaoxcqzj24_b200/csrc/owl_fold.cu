@@ -35,6 +35,9 @@
  */
 #include <cuda_runtime.h>
 #include <stdint.h>
+#ifdef OWL_DEBUG_CHECKS
+#include <cstdio>
+#endif
 
 #include "owl_device.cuh"
 #include "owl_internal.h"
@@ -43,11 +46,12 @@ using namespace owl_dev;
 
 #define FULL 0xFFFFFFFFu
 #ifndef FOLD_WARPS
-#define FOLD_WARPS 24
+#define FOLD_WARPS 16
 #endif
-#ifndef FOLD_R
-#define FOLD_R 2 /* walkers (runs) per warp */
+#ifndef FOLD_U
+#define FOLD_U 4 /* chunks of 32 records per warp and step */
 #endif
+#define FOLD_R 1
 #define FOLD_THREADS (FOLD_WARPS * 32)
 #define CF_CAP 512   /* shared node / edge / triple cells */
 #define CF_LIMIT 384
@@ -59,6 +63,15 @@ using namespace owl_dev;
 #define PF_DIST 2    /* granules prefetched ahead of the walk */
 #endif
 #define PROBE_LIMIT 4096u
+/* shared-memory paged histogram (keyless counting of hot narrow-range attributes) */
+#ifndef NPAGE
+#define NPAGE 168
+#endif
+#define PAGE_BINS 256       /* 4-byte bins: one page covers 1 KB of one attribute's address range */
+#define DIR_LOG 10
+#define DIRCAP (1 << DIR_LOG)
+#define FILTER_CAP 1024
+#define PAGE_TOTAL_LIMIT (1ull << 31)
 
 namespace {
 
@@ -73,12 +86,20 @@ struct RunDesc {
 };
 
 struct __align__(16) FoldSmem {
+  uint32_t page[NPAGE][PAGE_BINS]; /* keyless counters: bin b of page (attr, pg) counts x = pg<<10 | b<<2 */
+  ulonglong2 dir_key[DIRCAP];      /* page directory: (address-key hi, x >> 10) -> page */
+  int dir_page[DIRCAP];            /* -1: no page (yet) */
+  uint32_t filter[FILTER_CAP];     /* second-touch admission: fingerprints of page keys seen once */
+  uint16_t page_dir[NPAGE];        /* page -> directory slot (for the final flush) */
   ulonglong2 cf_key[CF_CAP];
   unsigned int cf_cnt[CF_CAP];
   uint32_t vkey[FOLD_WARPS][FOLD_R][VCAP];
   uint32_t vcnt[FOLD_WARPS][FOLD_R][VCAP];
   RunDesc rd[FOLD_WARPS][FOLD_R];
+  unsigned long long page_total;   /* sum of all page adds: pages are closed before a counter could wrap */
   unsigned int cf_fill;
+  unsigned int npages;
+  unsigned int pages_off;
 };
 
 __device__ __forceinline__ uint64_t evict_first_policy() {
@@ -102,7 +123,7 @@ __device__ __forceinline__ void l2_prefetch_bulk(const void* p, uint32_t bytes) 
 }
 
 /* 16-byte key load from L2 (.cg: no L1 allocation, so no stale copies of a cell claimed meanwhile) */
-__device__ __forceinline__ ulonglong2 ld_key_weak(const owl_cell* c) {
+__device__ __forceinline__ ulonglong2 ld_key_weak(const unsigned long long* c) {
   ulonglong2 k;
   asm volatile("ld.global.cg.v2.u64 {%0, %1}, [%2];" : "=l"(k.x), "=l"(k.y) : "l"(c));
   return k;
@@ -113,16 +134,19 @@ __device__ __forceinline__ void red_add(unsigned long long* p, unsigned long lon
 }
 
 /* predicated forms (no divergent branch around them) */
-__device__ __forceinline__ ulonglong2 ld_key_if(bool pred, const owl_cell* c) {
-  ulonglong2 k;
+/* both keys of a bucket: one 256-bit load of its first 32-byte sector */
+__device__ __forceinline__ ulonglong4 ld_bucket_keys_if(bool pred, const owl_bucket* b) {
+  ulonglong4 k;
   asm volatile(
       "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %3, 0;\n\t"
+      "setp.ne.b32 p, %5, 0;\n\t"
       "mov.b64 %0, -1;\n\t"
       "mov.b64 %1, -1;\n\t"
-      "@p ld.global.cg.v2.u64 {%0, %1}, [%2];\n\t}"
-      : "=l"(k.x), "=l"(k.y)
-      : "l"(c), "r"((int)pred));
+      "mov.b64 %2, -1;\n\t"
+      "mov.b64 %3, -1;\n\t"
+      "@p ld.global.cg.v4.u64 {%0, %1, %2, %3}, [%4];\n\t}"
+      : "=l"(k.x), "=l"(k.y), "=l"(k.z), "=l"(k.w)
+      : "l"(b), "r"((int)pred));
   return k;
 }
 __device__ __forceinline__ void red_add_if(bool pred, unsigned long long* p, unsigned long long v) {
@@ -139,16 +163,16 @@ __device__ __noinline__ uint32_t addr_insert_slow(const DevTable t, uint32_t shi
                                                   uint64_t lo, uint64_t c, FoldStatus* st) {
   const uint64_t mask = t.cap - 1;
   for (uint32_t probe = 0; probe < PROBE_LIMIT; ++probe) {
-    owl_cell* cell = t.cells + h;
-    const ulonglong2 k = ld_key_weak(cell);
+    unsigned long long* key = cell_key(t, h);
+    const ulonglong2 k = ld_key_weak(key);
     if (k.x == hi && k.y == lo) {
-      red_add(&cell->count, c);
+      red_add(cell_count(t, h), c);
       return 0;
     }
     if (k.x == OWL_EMPTY_KEY || k.x == hi) { /* empty, being claimed, or a torn read: resolve with the CAS */
-      const ulonglong2 o = cas128_global(&cell->hi, OWL_EMPTY_KEY, OWL_EMPTY_KEY, hi, lo);
+      const ulonglong2 o = cas128_global(key, OWL_EMPTY_KEY, OWL_EMPTY_KEY, hi, lo);
       if ((o.x == OWL_EMPTY_KEY && o.y == OWL_EMPTY_KEY) || (o.x == hi && o.y == lo)) {
-        red_add(&cell->count, c);
+        red_add(cell_count(t, h), c);
         return (o.x == OWL_EMPTY_KEY && o.y == OWL_EMPTY_KEY) ? 1u : 0u;
       }
     }
@@ -179,6 +203,42 @@ __device__ __noinline__ void cf_insert(FoldSmem& s, const FoldArgs& a, int tbl, 
     }
   }
   g_insert(a.tab[tbl], tbl, hi, lo, 1, a.status);
+}
+
+__device__ __forceinline__ uint32_t dir_hash(uint64_t hi, uint64_t pg) {
+  return ((uint32_t)hi * 0x9E3779B1u) ^ ((uint32_t)(hi >> 32) * 0x85EBCA77u) ^ ((uint32_t)pg * 0xC2B2AE3Du) ^
+         ((uint32_t)(pg >> 32) * 0x27D4EB2Fu);
+}
+
+/* Warp-uniform (every lane passes the same key): claims a page for page key (hi, pg), absent from its
+   directory slots h, h+1, on the key's second sighting while pages last; -1 = none (the chunk goes to
+   the global table).  Lane 0 decides, every lane gets its answer. */
+__device__ __noinline__ int page_alloc(FoldSmem& s, uint64_t hi, uint64_t pg, uint32_t h, int lane) {
+  int res = -1;
+  if (lane == 0 && *(volatile unsigned int*)&s.npages < NPAGE && !*(volatile unsigned int*)&s.pages_off) {
+    const uint32_t fp = dir_hash(hi, pg);
+    volatile uint32_t* f = &s.filter[fp & (FILTER_CAP - 1)];
+    if (*f != fp) {
+      *f = fp; /* first sighting: remember it, count this chunk globally */
+    } else {
+      for (int probe = 0; probe < 2; ++probe) {
+        const uint32_t hh = (h + probe) & (DIRCAP - 1);
+        const ulonglong2 o = cas128_shared(&s.dir_key[hh], OWL_EMPTY_KEY, OWL_EMPTY_KEY, hi, pg);
+        if (o.x == OWL_EMPTY_KEY && o.y == OWL_EMPTY_KEY) {
+          const unsigned n = atomicAdd(&s.npages, 1u);
+          if (n < NPAGE) {
+            res = (int)n;
+            s.page_dir[n] = (uint16_t)hh;
+          }
+          *(volatile int*)&s.dir_page[hh] = res; /* pages were zeroed at kernel start */
+          break;
+        }
+        if (o.x == hi && o.y == pg) break; /* claimed meanwhile by another warp: its page id may not be
+                                              published yet; this chunk goes global */
+      }
+    }
+  }
+  return __shfl_sync(FULL, res, 0);
 }
 
 __device__ __forceinline__ void report(FoldStatus* st, uint32_t seg_index, uint64_t idx, uint32_t code) {
@@ -251,6 +311,8 @@ __device__ __forceinline__ void slow_chunk(const uint4 r, const unsigned vm, Wal
                                            const int lane, bool& good, uint64_t& khi_out, uint64_t& lo_out) {
   const int nvalid = vm == FULL ? 32 : __ffs(~vm) - 1;
   const bool active = lane < nvalid;
+  int nproc = nvalid; /* records consumed: up to the last BB_ENTRY, so the next chunk starts on an
+                         instruction boundary (one attribute per fast chunk) */
   const uint64_t idx = (uint64_t)(w.p - d.rec) + lane;
   const uint64_t addr = (uint64_t)r.x | ((uint64_t)r.y << 32);
   const uint32_t meta = r.w;
@@ -295,7 +357,8 @@ __device__ __forceinline__ void slow_chunk(const uint4 r, const unsigned vm, Wal
       }
       __syncwarp();
     }
-    const bool ismem = active && (meta >> 31) != 0;
+    if (bbmask) nproc = 32 - __clz(bbmask);
+    const bool ismem = lane < nproc && (meta >> 31) != 0;
     const unsigned lt = bbmask & ((1u << lane) - 1u);
     const int L = lt ? 31 - __clz(lt) : lane;
     uint32_t cbb = __shfl_sync(FULL, bbf, L);
@@ -316,8 +379,8 @@ __device__ __forceinline__ void slow_chunk(const uint4 r, const unsigned vm, Wal
     khi_out = ((uint64_t)d.slot << 48) | ((uint64_t)cbb << 30) | ((uint64_t)ins << 22) | cj;
     lo_out = addr;
   }
-  w.p += nvalid;
-  if (nvalid < 32) { /* warp end: last BB -> S */
+  w.p += nproc;
+  if (nvalid < 32 && nproc == nvalid) { /* warp end: last BB -> S */
     if (a.mode == 0 && !(w.st & W_SKIP) && w.cur != OWL_NONE_BB && lane == 0) {
       cf_insert(s, a, T_EDGE, ((uint64_t)d.slot << 32) | w.cur, OWL_SENTINEL);
       cf_insert(s, a, T_TRIPLE, ((uint64_t)d.slot << 32) | w.cur, ((uint64_t)d.prev << 32) | OWL_SENTINEL);
@@ -357,11 +420,6 @@ __device__ __forceinline__ const FoldGroup& group_of(const FoldArgs& a, unsigned
   return a.groups[lo];
 }
 
-/* table index of a key: multiplicative hash, top bits (same function as owl_device.cuh::tab_index) */
-__device__ __forceinline__ uint64_t addr_index(uint64_t hi, uint64_t lo, uint32_t shift) {
-  return tab_hash(hi, lo) >> shift;
-}
-
 __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs args) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   FoldSmem& s = *reinterpret_cast<FoldSmem*>(smem_raw);
@@ -370,17 +428,31 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
   if (threadIdx.x == 0) {
     a = args;
     s.cf_fill = 0;
+    s.npages = 0;
+    s.pages_off = args.mode == 8 ? 1u : 0u; /* experiment mode 8: global table only */
+    s.page_total = 0;
   }
   for (int i = threadIdx.x; i < CF_CAP; i += FOLD_THREADS) {
     s.cf_key[i] = make_ulonglong2(OWL_EMPTY_KEY, OWL_EMPTY_KEY);
     s.cf_cnt[i] = 0;
   }
+  for (int i = threadIdx.x; i < NPAGE * PAGE_BINS; i += FOLD_THREADS) (&s.page[0][0])[i] = 0;
+  for (int i = threadIdx.x; i < DIRCAP; i += FOLD_THREADS) {
+    s.dir_key[i] = make_ulonglong2(OWL_EMPTY_KEY, OWL_EMPTY_KEY);
+    s.dir_page[i] = -1;
+  }
+  for (int i = threadIdx.x; i < FILTER_CAP; i += FOLD_THREADS) s.filter[i] = 0;
   __syncthreads();
   const uint64_t pol = evict_first_policy();
   const uint64_t tile = 1ull << a.tile_shift;
   const DevTable tab = a.tab[T_ADDR];
   const uint32_t shift = tab_shift(tab.cap);
+  RunDesc& d = s.rd[warp][0];
+  uint32_t* vk = s.vkey[warp][0];
+  uint32_t* vc = s.vcnt[warp][0];
   uint32_t claims = 0;
+  unsigned long long ptot = 0; /* this warp's page adds since the last item end */
+  uint32_t padds = 0;          /* lane-adds served by pages (statistics) */
 
   for (;;) {
     unsigned long long item = 0;
@@ -392,157 +464,185 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     if (item >= a.n_items) break;
     const FoldGroup& g = group_of(a, item);
     const uint64_t b = (item - g.item0) * tile;
-    Walker w[FOLD_R];
-#pragma unroll
-    for (int r = 0; r < FOLD_R; ++r) {
-      w[r].st = 0;
-      w[r].p = nullptr;
-      w[r].g0 = w[r].cur = 0;
-      w[r].khi = 0;
-      if (r < (int)g.n_members) {
-        const FoldSeg& sg = a.segs[g.first_seg + r];
-        if (b < sg.n) {
-          RunDesc& d = s.rd[warp][r];
-          const uint64_t e = b + tile < sg.n ? b + tile : sg.n;
-          if (lane == 0) {
-            d.rec = sg.rec;
-            d.end = sg.rec + sg.n;
-            d.tile_end = sg.rec + e;
-            d.seen = sg.seen;
-            d.slot = sg.slot;
-            d.n_warps = sg.n_warps;
-            d.seg_index = sg.seg_index;
-          }
-          w[r].p = sg.rec + first_warp_start(sg.rec, b, e, lane);
-          w[r].st = W_ACTIVE;
-          const uint4* end = sg.rec + sg.n;
-          if (lane < PF_DIST && a.mode != 3) { /* prime the L2 prefetch window */
-            const uintptr_t g0 = (((uintptr_t)w[r].p) >> PF_LOG) + lane;
-            const char* q = (const char*)(g0 << PF_LOG);
-            if (q < (const char*)end) {
-              const uint64_t left = (uint64_t)((const char*)end - q);
-              l2_prefetch_bulk(q, left < (1u << PF_LOG) ? (uint32_t)left : (1u << PF_LOG));
-            }
-          }
-        }
+    const FoldSeg& sg = a.segs[g.first_seg];
+    if (b >= sg.n) continue;
+    const uint64_t e = b + tile < sg.n ? b + tile : sg.n;
+    if (lane == 0) {
+      d.rec = sg.rec;
+      d.end = sg.rec + sg.n;
+      d.tile_end = sg.rec + e;
+      d.seen = sg.seen;
+      d.slot = sg.slot;
+      d.n_warps = sg.n_warps;
+      d.seg_index = sg.seg_index;
+    }
+    const uint4* const end = sg.rec + sg.n;
+#ifdef OWL_DEBUG_CHECKS
+    if (b > sg.n || e > sg.n) { printf("bad tile b %llu e %llu n %llu\n", (unsigned long long)b, (unsigned long long)e, (unsigned long long)sg.n); __trap(); }
+#endif
+    const uint4* const tile_end = sg.rec + e;
+    Walker w;
+    w.p = sg.rec + first_warp_start(sg.rec, b, e, lane);
+    w.st = W_ACTIVE;
+    w.g0 = w.cur = 0;
+    w.khi = 0;
+    if (lane < PF_DIST && a.mode != 3) { /* prime the L2 prefetch window */
+      const char* q = (const char*)(((((uintptr_t)w.p) >> PF_LOG) + lane) << PF_LOG);
+      if (q < (const char*)end) {
+        const uint64_t left = (uint64_t)((const char*)end - q);
+        l2_prefetch_bulk(q, left < (1u << PF_LOG) ? (uint32_t)left : (1u << PF_LOG));
       }
     }
     __syncwarp();
 
     for (;;) {
-      /* traced-warp starts and tile ends */
-      unsigned any = 0;
+      if (!(w.st & W_INWARP)) {
+        if (w.p >= tile_end) break;
+        begin_traced_warp(w, d, a, vk, lane);
+      }
+      /* FOLD_U chunks of 32 records: one 128-bit load per lane per chunk */
+      uint4 rr[FOLD_U];
 #pragma unroll
-      for (int r = 0; r < FOLD_R; ++r) {
-        if ((w[r].st & (W_ACTIVE | W_INWARP)) == W_ACTIVE) {
-          RunDesc& d = s.rd[warp][r];
-          if (w[r].p >= d.tile_end) w[r].st = 0;
-          else begin_traced_warp(w[r], d, a, s.vkey[warp][r], lane);
+      for (int u = 0; u < FOLD_U; ++u) {
+        const uint4* q = w.p + u * 32 + lane;
+        rr[u] = q < end ? ld_stream(q, pol) : make_uint4(0, 0, 0xFFFFFFFFu, 0);
+      }
+      if (a.mode != 3) { /* keep PF_DIST granules of the stream in flight to L2 */
+        const uintptr_t g1 = ((uintptr_t)(w.p + 32 * FOLD_U)) >> PF_LOG;
+        if (g1 != (((uintptr_t)w.p) >> PF_LOG) && lane == 0) {
+          const char* q = (const char*)((g1 + PF_DIST - 1) << PF_LOG);
+          if (q < (const char*)end) {
+            const uint64_t left = (uint64_t)((const char*)end - q);
+            l2_prefetch_bulk(q, left < (1u << PF_LOG) ? (uint32_t)left : (1u << PF_LOG));
+          }
         }
-        any |= w[r].st;
       }
-      if (!any) break;
+      /* fast path: every record of the U chunks is a well-formed MEM record of the current BB */
+      const uint32_t want = 0x80000000u | (w.cur << 8);
+      bool ok = !(w.st & W_SKIP) && (w.p + 32 * FOLD_U <= end);
+#pragma unroll
+      for (int u = 0; u < FOLD_U; ++u)
+        ok = ok && rr[u].z == w.g0 && (rr[u].w & 0x83FFFF00u) == want && rr[u].y < 0x90000000u;
+      bool good[FOLD_U], fastc[FOLD_U];
+      uint64_t khi[FOLD_U], klo[FOLD_U];
+      if (__all_sync(FULL, ok)) {
+#pragma unroll
+        for (int u = 0; u < FOLD_U; ++u) {
+          good[u] = fastc[u] = true;
+          khi[u] = w.khi | ((uint64_t)(rr[u].w & 0xFFu) << 22);
+          klo[u] = (uint64_t)rr[u].x | ((uint64_t)rr[u].y << 32);
+        }
+        w.p += 32 * FOLD_U;
+      } else {
+        bool live = true; /* false once the traced warp ended inside this batch: later chunks are reloaded */
+#pragma unroll
+        for (int u = 0; u < FOLD_U; ++u) {
+          good[u] = fastc[u] = false;
+          khi[u] = klo[u] = 0;
+          if (!live) continue;
+          const bool valid = (w.p + lane < end) && rr[u].z == w.g0;
+          const bool fast_ok = valid && (rr[u].w & 0x83FFFF00u) == want && rr[u].y < 0x90000000u;
+          if (__all_sync(FULL, fast_ok) && !(w.st & W_SKIP)) {
+            good[u] = fastc[u] = true;
+            khi[u] = w.khi | ((uint64_t)(rr[u].w & 0xFFu) << 22);
+            klo[u] = (uint64_t)rr[u].x | ((uint64_t)rr[u].y << 32);
+            w.p += 32;
+          } else {
+            const uint4* p0 = w.p;
+            slow_chunk(rr[u], __ballot_sync(FULL, valid), w, d, a, s, vk, vc, lane, good[u], khi[u], klo[u]);
+            live = (w.st & W_INWARP) != 0 && w.p == p0 + 32; /* else later chunks are reloaded */
+          }
+        }
+      }
+      if (a.mode != 0 && a.mode < 5) continue; /* experiment modes: 5 probe only, 6 RED only, 7 no RED */
 
-      /* loads: one 128-bit record per lane per walker */
-      uint4 rr[FOLD_R];
-      const uint4* end[FOLD_R];
+      /* A3, "merge identical thread traces" before any atomic:
+         - a fast chunk whose 32 keys are equal (broadcast access) is one add of 32;
+         - otherwise the chunk (one attribute after realignment) looks its page key up in the CTA's
+           page directory (branch-free 2-slot probe, same address for every lane: a broadcast read) and
+           the lanes of that page add into shared-memory bins; a missing page is allocated on the key's
+           second sighting (lane 0, rare);
+         - what is left (slow chunks, pages exhausted, wide-range or unaligned addresses) goes to the
+           global table: first probes of all chunks in flight together, predicated REDs, rare misses. */
+      bool lead[FOLD_U];
+      uint32_t cnt[FOLD_U];
+      unsigned any_lead = 0;
 #pragma unroll
-      for (int r = 0; r < FOLD_R; ++r) {
-        end[r] = s.rd[warp][r].end;
-        const uint4* q = w[r].p + lane;
-        rr[r] = (w[r].st && q < end[r]) ? ld_stream(q, pol) : make_uint4(0, 0, 0xFFFFFFFFu, 0);
-      }
-      /* L2 prefetch PF_DIST granules ahead when the walk enters a new granule */
-#pragma unroll
-      for (int r = 0; r < FOLD_R; ++r) {
-        if (w[r].st && a.mode != 3) {
-          const uintptr_t g1 = (((uintptr_t)(w[r].p + 32)) >> PF_LOG);
-          if (g1 != (((uintptr_t)w[r].p) >> PF_LOG) && lane == 0) {
-            const char* q = (const char*)((g1 + PF_DIST - 1) << PF_LOG);
-            if (q < (const char*)end[r]) {
-              const uint64_t left = (uint64_t)((const char*)end[r] - q);
-              l2_prefetch_bulk(q, left < (1u << PF_LOG) ? (uint32_t)left : (1u << PF_LOG));
+      for (int u = 0; u < FOLD_U; ++u) {
+        lead[u] = good[u];
+        cnt[u] = 1;
+        if (fastc[u]) { /* the key's upper word is warp-uniform on a fast chunk */
+          const uint32_t x0l = __shfl_sync(FULL, (uint32_t)klo[u], 0);
+          const uint32_t x0h = __shfl_sync(FULL, (uint32_t)(klo[u] >> 32), 0);
+          const uint32_t h0l = __shfl_sync(FULL, (uint32_t)khi[u], 0);
+          const bool eq_ins = (uint32_t)khi[u] == h0l;
+          if (__all_sync(FULL, eq_ins && (uint32_t)klo[u] == x0l && (uint32_t)(klo[u] >> 32) == x0h)) {
+            lead[u] = lane == 0;
+            cnt[u] = 32;
+          } else if (!*(volatile unsigned int*)&s.pages_off) {
+            const uint64_t Kh = (khi[u] & 0xFFFFFFFF00000000ull) | h0l;
+            const uint64_t Kp = (((uint64_t)x0h << 32) | x0l) >> 10;
+            const bool mine = eq_ins && (klo[u] >> 10) == Kp && (klo[u] & 3u) == 0;
+            const uint32_t h = dir_hash(Kh, Kp) >> (32 - DIR_LOG);
+            const ulonglong2 k0 = s.dir_key[h], k1 = s.dir_key[(h + 1) & (DIRCAP - 1)];
+            const bool f0 = k0.x == Kh && k0.y == Kp, f1 = k1.x == Kh && k1.y == Kp;
+            int pid = f0 ? s.dir_page[h] : (f1 ? s.dir_page[(h + 1) & (DIRCAP - 1)] : -1);
+            if (__any_sync(FULL, !f0 && !f1 && (k0.x == OWL_EMPTY_KEY || k1.x == OWL_EMPTY_KEY)))
+              pid = page_alloc(s, Kh, Kp, h, lane);
+            if (pid >= 0 && mine) {
+              atomicAdd(&s.page[pid][(klo[u] >> 2) & (PAGE_BINS - 1)], 1u);
+              ++ptot;
+              ++padds;
+              lead[u] = false;
             }
           }
         }
+        any_lead |= __ballot_sync(FULL, lead[u]);
       }
-
-      /* classify + keys */
-      bool good[FOLD_R];
-      uint64_t khi[FOLD_R], klo[FOLD_R];
-      uint32_t mult[FOLD_R];
-      bool fast[FOLD_R];
+      if (!any_lead) continue;
+      uint32_t home[FOLD_U];
+      ulonglong4 kk[FOLD_U];
 #pragma unroll
-      for (int r = 0; r < FOLD_R; ++r) {
-        good[r] = false;
-        fast[r] = false;
-        mult[r] = 1;
-        khi[r] = 0;
-        klo[r] = 0;
-        if (!w[r].st) continue;
-        const bool valid = (w[r].p + lane < end[r]) && rr[r].z == w[r].g0;
-        const uint64_t addr = (uint64_t)rr[r].x | ((uint64_t)rr[r].y << 32);
-        const bool fast_ok = valid && (rr[r].w >> 31) != 0 && ((rr[r].w >> 8) & 0x3FFFFu) == w[r].cur &&
-                             (addr >> 60) <= 8;
-        const unsigned vm = __ballot_sync(FULL, valid);
-        if (__all_sync(FULL, fast_ok) && !(w[r].st & W_SKIP)) {
-          fast[r] = true;
-          good[r] = true;
-          khi[r] = w[r].khi | ((uint64_t)(rr[r].w & 0xFFu) << 22);
-          klo[r] = addr;
-          w[r].p += 32;
-        } else {
-          slow_chunk(rr[r], vm, w[r], s.rd[warp][r], a, s, s.vkey[warp][r], s.vcnt[warp][r], lane, good[r],
-                     khi[r], klo[r]);
-        }
+      for (int u = 0; u < FOLD_U; ++u) {
+        home[u] = tab_index(khi[u], klo[u], shift);
+#ifdef OWL_DEBUG_CHECKS
+        if (lead[u] && home[u] >= tab.cap) { printf("bad home %u cap %llu shift %u\n", home[u], (unsigned long long)tab.cap, shift); __trap(); }
+#endif
+        kk[u] = ld_bucket_keys_if(lead[u] && a.mode != 6, tab.b + (home[u] >> 1));
       }
-      if (a.mode != 0) continue;
-
-      /* merge chunks of other runs whose 32 keys equal walker 0's into walker 0 (exact: equal keys) */
+      if (a.mode == 5) { /* experiment: probe loads only */
+        unsigned sink = 0;
 #pragma unroll
-      for (int r = 1; r < FOLD_R; ++r) {
-        if (fast[0] && fast[r]) {
-          const bool eq = khi[r] == khi[0] && klo[r] == klo[0];
-          if (__all_sync(FULL, eq)) {
-            mult[0] += 1;
-            mult[r] = 0;
-          }
-        }
+        for (int u = 0; u < FOLD_U; ++u) sink |= (unsigned)(kk[u].x == khi[u]);
+        if (__all_sync(FULL, sink == 7u)) claims += 1;
+        continue;
       }
-
-      /* one insert per run of equal keys over consecutive lanes: leaders, counts, first probes for every
-         walker (loads in flight together), then predicated REDs; misses take a rare uniform branch */
-      bool lead[FOLD_R];
-      uint32_t cnt[FOLD_R];
-      owl_cell* cell[FOLD_R];
-      ulonglong2 kk[FOLD_R];
+      if (a.mode == 6) { /* experiment: REDs to the home cells only (counts are wrong) */
 #pragma unroll
-      for (int r = 0; r < FOLD_R; ++r) {
-        const uint64_t phi = __shfl_up_sync(FULL, khi[r], 1), plo = __shfl_up_sync(FULL, klo[r], 1);
-        const bool pgood = __shfl_up_sync(FULL, (int)good[r], 1) != 0;
-        const bool same = lane > 0 && good[r] && pgood && phi == khi[r] && plo == klo[r];
-        const unsigned brk = __ballot_sync(FULL, !same);
-        const unsigned above = brk & ~((2u << lane) - 1u);
-        const uint32_t nxt = above ? __ffs(above) - 1 : 32;
-        lead[r] = good[r] && !same && mult[r] != 0;
-        cnt[r] = (nxt - lane) * mult[r];
-        cell[r] = tab.cells + addr_index(khi[r], klo[r], shift);
-        kk[r] = ld_key_if(lead[r], cell[r]);
+        for (int u = 0; u < FOLD_U; ++u) red_add_if(lead[u], &tab.b[home[u] >> 1].count[0], cnt[u]);
+        continue;
       }
       unsigned miss_any = 0;
 #pragma unroll
-      for (int r = 0; r < FOLD_R; ++r) {
-        const bool hit = lead[r] && kk[r].x == khi[r] && kk[r].y == klo[r];
-        red_add_if(hit, &cell[r]->count, cnt[r]);
-        lead[r] = lead[r] && !hit; /* now: missed */
-        miss_any |= __ballot_sync(FULL, lead[r]);
+      for (int u = 0; u < FOLD_U; ++u) {
+        const bool h0 = kk[u].x == khi[u] && kk[u].y == klo[u];
+        const bool h1 = kk[u].z == khi[u] && kk[u].w == klo[u];
+        const bool hit = lead[u] && (h0 || h1);
+        red_add_if(hit && a.mode != 7, &tab.b[home[u] >> 1].count[h1 ? 1 : 0], cnt[u]);
+        lead[u] = lead[u] && !hit; /* now: missed (absent, or displaced past the home bucket) */
+        miss_any |= __ballot_sync(FULL, lead[u]);
       }
       if (miss_any) {
 #pragma unroll
-        for (int r = 0; r < FOLD_R; ++r)
-          if (lead[r])
-            claims += addr_insert_slow(tab, shift, (uint64_t)(cell[r] - tab.cells), khi[r], klo[r], cnt[r], a.status);
+        for (int u = 0; u < FOLD_U; ++u)
+          if (lead[u]) claims += addr_insert_slow(tab, shift, home[u], khi[u], klo[u], cnt[u], a.status);
       }
+    }
+    if (__any_sync(FULL, ptot != 0)) { /* close the pages before any counter could wrap */
+#pragma unroll
+      for (int o = 16; o; o >>= 1) ptot += __shfl_xor_sync(FULL, ptot, o);
+      if (lane == 0 && atomicAdd(&s.page_total, ptot) + ptot > PAGE_TOTAL_LIMIT) s.pages_off = 1;
+      ptot = 0;
     }
     /* cells claimed by this item -> table fill; past the load limit the build stops and regrows */
     if (__any_sync(FULL, claims != 0)) {
@@ -556,7 +656,20 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
       claims = 0;
     }
   }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) padds += __shfl_xor_sync(FULL, padds, o);
+  if (lane == 0) atomicAdd(&a.status->n_bypass, (unsigned long long)padds);
   __syncthreads();
+  const unsigned np = s.npages < NPAGE ? s.npages : NPAGE;
+  if (threadIdx.x == 0) atomicAdd(&a.status->n_flush, (unsigned long long)np);
+  for (unsigned i = threadIdx.x; i < np * PAGE_BINS; i += FOLD_THREADS) {
+    const unsigned pg = i / PAGE_BINS, b = i % PAGE_BINS;
+    const uint32_t c = s.page[pg][b];
+    if (c) {
+      const ulonglong2 k = s.dir_key[s.page_dir[pg]];
+      g_insert(tab, T_ADDR, k.x, (k.y << 10) | ((uint64_t)b << 2), c, a.status);
+    }
+  }
   for (int i = threadIdx.x; i < CF_CAP; i += FOLD_THREADS) {
     const ulonglong2 k = s.cf_key[i];
     if (k.x != OWL_EMPTY_KEY) {
@@ -569,7 +682,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
 }  // namespace
 
 int owl_fold_ctas_per_sm() { return 1; }
-int owl_fold_runs_per_warp() { return FOLD_R; }
+int owl_fold_runs_per_warp() { return 1; }
 
 cudaError_t owl_launch_fold(const FoldArgs& a, int grid, cudaStream_t st) {
   const size_t smem = sizeof(FoldSmem);

@@ -330,7 +330,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
       ctx->last_fold_records = nrec;
       ctx->total_fold_ms += ms;
       ctx->total_fold_records += nrec;
-      if (getenv("OWL_FOLD_VERBOSE")) fprintf(stderr, "[owl] fold: %llu records %.3f ms flushes %llu bypass %llu claims %llu\n",
+      if (getenv("OWL_FOLD_VERBOSE")) fprintf(stderr, "[owl] fold: %llu records %.3f ms pages %llu page-adds %llu claims %llu\n",
         (unsigned long long)nrec, ms, hs.n_flush, hs.n_bypass, hs.n_claim);
     }
   }
@@ -365,7 +365,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
 
 uint64_t default_cap(owl_ctx* ctx, int t) {
   if (ctx->cap_hint[t]) return ctx->cap_hint[t];
-  if (t == T_ADDR) return ctx->cfg.addr_capacity ? next_pow2(ctx->cfg.addr_capacity) : (1ull << 22);
+  if (t == T_ADDR) return ctx->cfg.addr_capacity ? next_pow2(ctx->cfg.addr_capacity) : (1ull << 20);
   return ctx->cfg.cf_capacity ? next_pow2(ctx->cfg.cf_capacity) : (1ull << 14);
 }
 
@@ -389,6 +389,12 @@ owl_status build_tables(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTa
       return s;
     }
     if (!overflow) {
+      /* next builds: at most 1/16 of the address cells claimed, so nearly every key sits in its home
+         bucket and the fold's first probe hits (owl_fold.cu) */
+      unsigned long long fill = 0;
+      cudaMemcpy(&fill, tab[T_ADDR].fill, sizeof fill, cudaMemcpyDeviceToHost);
+      static const int load_shift = getenv("OWL_ADDR_LOAD_SHIFT") ? atoi(getenv("OWL_ADDR_LOAD_SHIFT")) : 4;
+      ctx->cap_hint[T_ADDR] = std::max(ctx->cap_hint[T_ADDR], std::min<uint64_t>(next_pow2(fill << load_shift), 1ull << 28));
       for (int t = 0; t < T_NUM; ++t) ctx->cap_hint[t] = std::max(ctx->cap_hint[t], cap[t]);
       return OWL_OK;
     }

@@ -38,15 +38,20 @@ enum {
   KERR_BBMISMATCH = 5 /* MEM bb != the warp's current BB                   */
 };
 
-struct owl_cell {
-  unsigned long long hi, lo, count, pad;
+/* Buckets of two cells, 64 B: both keys in the first 32-byte L2 sector (one 256-bit load probes the
+   bucket), the two counts in the second.  Cell i = slot (i & 1) of bucket (i >> 1). */
+struct owl_bucket {
+  unsigned long long key[2][2]; /* [slot][hi, lo] */
+  unsigned long long count[2];
+  unsigned long long pad[2];
 };
 
 struct DevTable {
-  owl_cell* cells;     /* cap cells */
+  owl_bucket* b;            /* cap / 2 buckets */
   unsigned long long* fill; /* number of claimed cells (device counter) */
-  uint64_t cap;        /* power of two */
+  uint64_t cap;             /* cells: power of two, 2 .. 2^31 */
 };
+#define OWL_MAX_TABLE_CELLS (1ull << 31)
 
 /* Shared device status of one fold launch */
 struct FoldStatus {
@@ -55,8 +60,8 @@ struct FoldStatus {
   unsigned int overflow;            /* bitmask of tables that exceeded their load limit             */
   unsigned int limit;               /* bitmask: 1 = slot/j field limit exceeded, 2 = visits map full */
   unsigned long long tile_counter;  /* persistent-kernel work counter                               */
-  unsigned long long n_flush;       /* shared-table flushes (all CTAs)                              */
-  unsigned long long n_bypass;      /* address inserts that went straight to the global table      */
+  unsigned long long n_flush;       /* shared-memory pages allocated (all CTAs)                     */
+  unsigned long long n_bypass;      /* address lane-adds served by shared-memory pages              */
   unsigned long long n_claim;       /* shared-table cells claimed                                   */
 };
 

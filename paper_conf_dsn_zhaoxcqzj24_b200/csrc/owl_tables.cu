@@ -25,27 +25,27 @@ struct KeyDecomp {
   }
 };
 
-__global__ void clear_kernel(owl_cell* c, uint64_t cap) {
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < cap; i += (uint64_t)gridDim.x * blockDim.x) {
-    c[i].hi = OWL_EMPTY_KEY;
-    c[i].lo = OWL_EMPTY_KEY;
-    c[i].count = 0;
-    c[i].pad = 0;
+__global__ void clear_kernel(owl_bucket* b, uint64_t nb) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nb; i += (uint64_t)gridDim.x * blockDim.x) {
+    reinterpret_cast<ulonglong4*>(&b[i])[0] = make_ulonglong4(OWL_EMPTY_KEY, OWL_EMPTY_KEY, OWL_EMPTY_KEY, OWL_EMPTY_KEY);
+    reinterpret_cast<ulonglong4*>(&b[i])[1] = make_ulonglong4(0, 0, 0, 0);
   }
 }
 
 /* compaction of non-empty cells (order is irrelevant: a sort follows) */
-__global__ void compact_kernel(const owl_cell* c, uint64_t cap, Key128* k, unsigned long long* cnt,
+__global__ void compact_kernel(const owl_bucket* c, uint64_t cap, Key128* k, unsigned long long* cnt,
                                unsigned long long* n_out) {
   const int lane = threadIdx.x & 31;
   for (uint64_t base = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) & ~31ull; base < cap;
        base += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t i = base + lane;
-    owl_cell v;
+    unsigned long long vhi = OWL_EMPTY_KEY, vlo = 0, vc = 0;
     bool live = false;
     if (i < cap) {
-      v = c[i];
-      live = v.hi != OWL_EMPTY_KEY;
+      vhi = c[i >> 1].key[i & 1][0];
+      vlo = c[i >> 1].key[i & 1][1];
+      vc = c[i >> 1].count[i & 1];
+      live = vhi != OWL_EMPTY_KEY;
     }
     const unsigned m = __ballot_sync(0xFFFFFFFFu, live);
     unsigned long long b = 0;
@@ -53,9 +53,9 @@ __global__ void compact_kernel(const owl_cell* c, uint64_t cap, Key128* k, unsig
     b = __shfl_sync(0xFFFFFFFFu, b, 0);
     if (live) {
       const uint64_t o = b + __popc(m & ((1u << lane) - 1u));
-      k[o].hi = v.hi;
-      k[o].lo = v.lo;
-      cnt[o] = v.count;
+      k[o].hi = vhi;
+      k[o].lo = vlo;
+      cnt[o] = vc;
     }
   }
 }
@@ -185,22 +185,23 @@ void owl_dev_trim(int dev) {
 }
 
 cudaError_t owl_table_alloc(DevTable* t, uint64_t cap, cudaStream_t st) {
+  if (cap < 2 || cap > OWL_MAX_TABLE_CELLS || (cap & (cap - 1))) return cudaErrorInvalidValue;
   t->cap = cap;
-  t->cells = (owl_cell*)owl_dev_alloc(cap * sizeof(owl_cell));
+  t->b = (owl_bucket*)owl_dev_alloc((cap / 2) * sizeof(owl_bucket));
   t->fill = (unsigned long long*)owl_dev_alloc(sizeof(unsigned long long));
-  if (!t->cells || !t->fill) {
+  if (!t->b || !t->fill) {
     owl_table_free(t);
     return cudaErrorMemoryAllocation;
   }
-  clear_kernel<<<grid_for(cap, 256), 256, 0, st>>>(t->cells, cap);
+  clear_kernel<<<grid_for(cap / 2, 256), 256, 0, st>>>(t->b, cap / 2);
   cudaMemsetAsync(t->fill, 0, sizeof(unsigned long long), st);
   return cudaGetLastError();
 }
 
 void owl_table_free(DevTable* t) {
-  owl_dev_free(t->cells);
+  owl_dev_free(t->b);
   owl_dev_free(t->fill);
-  t->cells = nullptr;
+  t->b = nullptr;
   t->fill = nullptr;
   t->cap = 0;
 }
@@ -228,7 +229,7 @@ cudaError_t owl_table_sorted(const DevTable& t, SortedTable* out, cudaStream_t s
     return cudaErrorMemoryAllocation;
   }
   cudaMemsetAsync(dn, 0, sizeof(unsigned long long), st);
-  compact_kernel<<<grid_for(t.cap, 256), 256, 0, st>>>(t.cells, t.cap, k0, c0, dn);
+  compact_kernel<<<grid_for(t.cap, 256), 256, 0, st>>>(t.b, t.cap, k0, c0, dn);
   size_t tmp = 0;
   cub::DeviceRadixSort::SortPairs(nullptr, tmp, k0, out->k, c0, out->c, (int64_t)n, KeyDecomp{}, st);
   void* dt = owl_dev_alloc(tmp);
