@@ -47,11 +47,12 @@ class ClockSampler:
 
     def __init__(self, index=0):
         self.index, self.rows, self.proc = index, [], None
+        self.window, self._seen = False, False
 
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                          "--format=csv,noheader,nounits", "-lms", "20"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -60,9 +61,16 @@ class ClockSampler:
 
     def _read(self):
         for line in self.proc.stdout:
+            self._seen = True
             parts = [x.strip() for x in line.split(",")]
-            if len(parts) >= 7:
+            if len(parts) >= 7 and self.window:
                 self.rows.append(parts)
+
+    def wait_ready(self, timeout=10.0):
+        """nvidia-smi needs ~0.5-1 s to start: wait until it prints, so the timed region is covered."""
+        t0 = time.time()
+        while self.proc and not self._seen and time.time() - t0 < timeout and self.proc.poll() is None:
+            time.sleep(0.05)
 
     def stop(self):
         if not self.proc:
@@ -283,15 +291,17 @@ def run_ours(args):
         er.destroy()
         tick("destroy", t0)
 
+    clocks = ClockSampler(local)
+    clocks.start()  # nvidia-smi starts up during the warm-up; only timed-region samples are kept
     for _ in range(args.warmup):
         step()
     brk.clear()
     ctx.reset_stats()
-    clocks = ClockSampler(local)
+    clocks.wait_ready()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    clocks.start()
+    clocks.window = True
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
     for _ in range(args.steps):
@@ -349,7 +359,7 @@ def run_ours(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", type=int, default=2, help="workload C1..C5 (default: configs[1], C2)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])

@@ -2,42 +2,38 @@
  * owl_fold.cu — A1-A3: stream trace records once and fold them thread -> warp -> kernel into the
  * A-DCFG hash tables (§V.A-B).
  *
- * Design (measurements in profiles/):
+ * Design v7 (measurements in profiles/): the fold is an HBM stream whose per-record work
+ * must fit the issue budget (≈5.5 warp-instructions per record at 50% of HBM on 148 SMs), so every choice
+ * below minimises instructions per 32-record chunk:
  *
- *  * persistent CTAs of FOLD_WARPS independent warps; a warp pops one work item at a time from a global
- *    counter.  A work item is (group, tile p): a group holds up to FOLD_R segments of one evidence slot
- *    (consecutive runs of one class), and the warp walks tile p of every member AT ONCE — FOLD_R walkers
- *    whose state is warp-uniform and lives in registers, one 128-bit record load per lane per walker and
- *    step, so FOLD_R x 512 B are in flight per warp besides the L2 bulk prefetch that runs ahead;
- *  * a tile holds the traced warps whose first record lies in it: a walker that starts inside a traced
- *    warp finds the next warp start with a 33-ary warp-cooperative search, and the walker that owns a
- *    traced warp finishes it past the tile end;
- *  * per traced warp a walker takes the records 32 at a time (one per lane):
- *      A2  fast path: 32 MEM records of the current basic block — the key of lane i is
- *          (slot, cur, ins_i, j, x_i); the context (cur, j) is warp-uniform.  Chunks holding a BB_ENTRY,
- *          a warp end or a malformed record take the slow path, which applies the BB entries in lane
- *          order with warp-uniform state (cur, prev, the per-warp visit ordinal j of each BB in a
- *          shared-memory map), counts node / edge / triple cells in a small shared-memory table,
- *          and gives every MEM lane the context of the last BB_ENTRY lane before it;
- *      A3  "merging identical thread traces" at two levels before any atomic:
- *          - across runs: a fast-path chunk of walker r that is bit-identical to walker 0's chunk under
- *            the same context (same slot, BB, visit) adds its counts to walker 0's (exact: the records
- *            and the context ARE the key) — every FIX run of a deterministic program folds as one;
- *          - across lanes: consecutive lanes with equal keys (broadcast loads) form one add of their
- *            count;
- *          then one insert per distinct key into the global open-addressing table (32-byte cells, one L2
- *          sector each): the key probe is a plain (L1-cacheable) load — keys are immutable once
- *          claimed, a stale "empty" only sends the lane to the 128-bit CAS — and the count update is a
- *          fire-and-forget RED.64 in L2, where the hot cells of a trace stay resident (the record stream
- *          is loaded L2::evict_first).
- * Malformed records are reported with the minimum (segment, index) and skipped (state unaffected), exactly
- * as the oracle does.
+ *  * persistent CTAs of FOLD_WARPS independent warps; a warp pops one work item (segment, tile of 2^k
+ *    records) at a time from a global counter.  A tile holds the traced warps whose first record lies in
+ *    it: the warp finds the first such start with a 33-ary warp-cooperative search and finishes the last
+ *    traced warp past the tile end;
+ *  * a warp walks its traced warp FOLD_U chunks of 32 records at a time (one 128-bit streaming load per
+ *    lane and chunk), with cp.async.bulk.prefetch.L2 keeping the next granules of its stream in flight;
+ *  * A2: a chunk whose 32 records are well-formed MEM records of the current basic block takes the fast
+ *    path (its context (cur, j) is warp-uniform).  A chunk holding a BB_ENTRY, a warp end or a malformed
+ *    record takes the slow path: it consumes records up to its last BB_ENTRY, applies the entries in lane
+ *    order with warp-uniform state (cur, prev, the per-warp visit ordinal j of each BB in a shared-memory
+ *    map), counts node / edge / triple cells in a shared-memory table, and gives every MEM lane
+ *    the context of the last BB_ENTRY lane before it.  The next chunk then starts on an instruction
+ *    boundary, so a fast chunk is normally one instruction executed by 32 threads;
+ *  * A3, "merging identical thread traces" before any global atomic.  A fast chunk is
+ *      - broadcast (32 equal keys): one add of 32 to its cell in the CTA's shared-memory directory;
+ *      - page-local (one attribute, one 1 KB window of addresses, 4-byte aligned — T-table lookups,
+ *        tiles of shared memory): each lane adds 1 to a keyless 4-byte bin of the window's shared-memory
+ *        page (pages are admitted on a window's second sighting while they last);
+ *      - otherwise (thread-distinct addresses, pages exhausted, slow-chunk lanes): one insert per lane
+ *        into the global open-addressing table, first probes of all chunks of the step in flight
+ *        together, counts added with fire-and-forget RED.64 in L2.
+ *    The shared directory / pages / CF cells are exact partial sums, flushed to the global tables when
+ *    the CTA finishes.
+ * Malformed records are reported with the minimum (segment, index) and skipped (state unaffected),
+ * exactly as the oracle does.
  */
 #include <cuda_runtime.h>
 #include <stdint.h>
-#ifdef OWL_DEBUG_CHECKS
-#include <cstdio>
-#endif
 
 #include "owl_device.cuh"
 #include "owl_internal.h"
@@ -51,11 +47,11 @@ using namespace owl_dev;
 #ifndef FOLD_U
 #define FOLD_U 4 /* chunks of 32 records per warp and step */
 #endif
-#define FOLD_R 1
 #define FOLD_THREADS (FOLD_WARPS * 32)
-#define CF_CAP 512   /* shared node / edge / triple cells */
-#define CF_LIMIT 384
-#define VCAP 128     /* per-walker visit map (distinct BBs of one traced warp) */
+#define CFK 128      /* shared cells per CF table kind (node, edge, triple) */
+#define CFK_LIMIT 96
+#define VCAP 128     /* per-warp visit map (distinct BBs of one traced warp) */
+#define VGEN_MAX 0x3FFFu /* visit-map entry = gen<<18 | bb: a new generation per traced warp, 0 = empty */
 #ifndef PF_LOG
 #define PF_LOG 12    /* L2 bulk prefetch granule: 4 KB (256 records) */
 #endif
@@ -63,43 +59,58 @@ using namespace owl_dev;
 #define PF_DIST 2    /* granules prefetched ahead of the walk */
 #endif
 #define PROBE_LIMIT 4096u
-/* shared-memory paged histogram (keyless counting of hot narrow-range attributes) */
 #ifndef NPAGE
 #define NPAGE 168
 #endif
-#define PAGE_BINS 256       /* 4-byte bins: one page covers 1 KB of one attribute's address range */
+#define PAGE_BINS 256 /* 4-byte bins: one page counts the 1 KB address window x>>10 of one attribute */
+#ifndef DIR_LOG
 #define DIR_LOG 10
+#endif
+#define FILTER_LOG 11 /* admission filter: sightings of keys not (yet) in the directory */
 #define DIRCAP (1 << DIR_LOG)
-#define FILTER_CAP 1024
-#define PAGE_TOTAL_LIMIT (1ull << 31)
+#define PAGE_TAG (3ull << 62) /* directory key lo of a page window: (x>>10) | PAGE_TAG (never a valid x) */
+/* directory value of a page window: PV_PAGE | page id, or no page (0 while being admitted, PV_NONE
+   once pages ran out); of a broadcast cell: its count */
+#ifndef ADMIT
+#define ADMIT 16u    /* a key enters the directory on its ADMIT-th sighting: recurring keys, not one-offs */
+#endif
+#define PV_NONE 0x40000000u
+#define PV_PAGE 0x80000000u
+/* a CTA stops using shared counters once it has walked this many records (every shared counter is
+   bounded by the records walked, so no 32-bit counter can wrap) */
+#define SHARED_TOTAL_LIMIT (1ull << 31)
+
+#ifdef OWL_FOLD_STATS
+#define STAT(i) (++stat[i])
+#else
+#define STAT(i) ((void)0)
+#endif
 
 namespace {
 
-/* per-walker fields read only at traced-warp / tile boundaries and on errors */
+/* per-warp fields read only at traced-warp / tile boundaries, in the slow path and on errors */
 struct RunDesc {
-  const uint4* rec;      /* segment base */
-  const uint4* end;      /* segment end */
-  const uint4* tile_end; /* traced warps starting at or after this belong to the next tile */
+  const uint4* rec; /* segment base */
   uint32_t* seen;
   uint32_t slot, n_warps, seg_index;
-  uint32_t prev, curj;   /* walk context read only by the slow path (cur and khi stay in registers) */
+  uint32_t prev, curj;
 };
 
 struct __align__(16) FoldSmem {
-  uint32_t page[NPAGE][PAGE_BINS]; /* keyless counters: bin b of page (attr, pg) counts x = pg<<10 | b<<2 */
-  ulonglong2 dir_key[DIRCAP];      /* page directory: (address-key hi, x >> 10) -> page */
-  int dir_page[DIRCAP];            /* -1: no page (yet) */
-  uint32_t filter[FILTER_CAP];     /* second-touch admission: fingerprints of page keys seen once */
-  uint16_t page_dir[NPAGE];        /* page -> directory slot (for the final flush) */
-  ulonglong2 cf_key[CF_CAP];
-  unsigned int cf_cnt[CF_CAP];
-  uint32_t vkey[FOLD_WARPS][FOLD_R][VCAP];
-  uint32_t vcnt[FOLD_WARPS][FOLD_R][VCAP];
-  RunDesc rd[FOLD_WARPS][FOLD_R];
-  unsigned long long page_total;   /* sum of all page adds: pages are closed before a counter could wrap */
-  unsigned int cf_fill;
+  uint32_t page[NPAGE][PAGE_BINS];
+  ulonglong2 dir_key[DIRCAP]; /* (attribute key hi, x) broadcast cell, or (hi, x>>10 | PAGE_TAG) window */
+  uint32_t dir_val[DIRCAP];
+  uint32_t filt[1 << FILTER_LOG]; /* 4-way buckets of tag<<8 | sightings of keys not in the directory */
+  uint32_t vkey[FOLD_WARPS][VCAP]; /* per-warp visit maps: gen<<18 | bb, and the visit count */
+  uint32_t vcnt[FOLD_WARPS][VCAP];
+  uint16_t page_dir[NPAGE];   /* page -> directory slot (final flush) */
+  ulonglong2 cf_key[3][CFK];  /* node / edge / triple cells, one table per kind */
+  unsigned int cf_cnt[3][CFK];
+  unsigned int cf_fill[3];
+  RunDesc rd[FOLD_WARPS];
+  unsigned long long walked; /* records walked by the CTA */
   unsigned int npages;
-  unsigned int pages_off;
+  unsigned int off;          /* 1: shared counting closed (total limit, or experiment mode 8) */
 };
 
 __device__ __forceinline__ uint64_t evict_first_policy() {
@@ -116,8 +127,7 @@ __device__ __forceinline__ uint4 ld_stream(const uint4* p, uint64_t pol) {
   return r;
 }
 
-/* L2 prefetch with normal eviction priority: the lines must survive until the walk's demand loads (which
-   then mark them evict_first) */
+/* L2 prefetch with normal eviction priority: the lines must survive until the walk's demand loads */
 __device__ __forceinline__ void l2_prefetch_bulk(const void* p, uint32_t bytes) {
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
 }
@@ -133,8 +143,7 @@ __device__ __forceinline__ void red_add(unsigned long long* p, unsigned long lon
   asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-/* predicated forms (no divergent branch around them) */
-/* both keys of a bucket: one 256-bit load of its first 32-byte sector */
+/* both keys of a bucket: one 256-bit load of its first 32-byte sector (predicated, no branch) */
 __device__ __forceinline__ ulonglong4 ld_bucket_keys_if(bool pred, const owl_bucket* b) {
   ulonglong4 k;
   asm volatile(
@@ -158,9 +167,10 @@ __device__ __forceinline__ void red_add_if(bool pred, unsigned long long* p, uns
       : "memory");
 }
 
-/* probe continuation of an address-cell insert whose first probe at `h` missed; returns cells claimed */
-__device__ __noinline__ uint32_t addr_insert_slow(const DevTable t, uint32_t shift, uint64_t h, uint64_t hi,
-                                                  uint64_t lo, uint64_t c, FoldStatus* st) {
+/* probe continuation of an address-cell insert whose first probe (home bucket) missed; returns cells
+   claimed */
+__device__ __noinline__ uint32_t addr_insert_slow(const DevTable t, uint64_t h, uint64_t hi, uint64_t lo,
+                                                  uint64_t c, FoldStatus* st) {
   const uint64_t mask = t.cap - 1;
   for (uint32_t probe = 0; probe < PROBE_LIMIT; ++probe) {
     unsigned long long* key = cell_key(t, h);
@@ -179,80 +189,81 @@ __device__ __noinline__ uint32_t addr_insert_slow(const DevTable t, uint32_t shi
     h = (h + 1) & mask;
   }
   atomicOr(&st->overflow, 1u << T_ADDR); /* pathological clustering: regrow */
-  (void)shift;
   return 0;
 }
 
-/* node / edge / triple cells (the table id rides in key bits 62-63; slot < 2^16) */
+/* node / edge / triple cell += 1 in the CTA's table of kind `tbl` (T_NODE / T_EDGE / T_TRIPLE); lanes of
+   one call may insert concurrently as long as they use different kinds (different arrays) */
 __device__ __noinline__ void cf_insert(FoldSmem& s, const FoldArgs& a, int tbl, uint64_t hi, uint64_t lo) {
-  const uint64_t thi = hi | ((uint64_t)tbl << 62);
-  if (*(volatile unsigned int*)&s.cf_fill < CF_LIMIT) {
-    uint32_t h = (uint32_t)(hmix(thi, lo) & (CF_CAP - 1));
-    for (int probe = 0; probe < CF_CAP; ++probe) {
-      const ulonglong2 o = cas128_shared(&s.cf_key[h], OWL_EMPTY_KEY, OWL_EMPTY_KEY, thi, lo);
-      if (o.x == OWL_EMPTY_KEY && o.y == OWL_EMPTY_KEY) {
-        atomicAdd(&s.cf_fill, 1u);
-        atomicAdd(&s.cf_cnt[h], 1u);
-        return;
-      }
-      if (o.x == thi && o.y == lo) {
-        atomicAdd(&s.cf_cnt[h], 1u);
-        return;
-      }
-      h = (h + 1) & (CF_CAP - 1);
+  ulonglong2* K = s.cf_key[tbl];
+  uint32_t h = (((uint32_t)hi * 0x9E3779B1u) ^ ((uint32_t)(hi >> 32) * 0x85EBCA77u) ^ ((uint32_t)lo * 0xC2B2AE3Du) ^
+                (uint32_t)(lo >> 32)) >> 25; /* CFK = 128 */
+  for (int probe = 0; probe < CFK; ++probe) {
+    const ulonglong2 k = K[h];
+    if (k.x == hi && k.y == lo) {
+      atomicAdd(&s.cf_cnt[tbl][h], 1u);
+      return;
     }
+    if (k.x == OWL_EMPTY_KEY) {
+      if (*(volatile unsigned int*)&s.cf_fill[tbl] >= CFK_LIMIT) break;
+      const ulonglong2 o = cas128_shared(&K[h], OWL_EMPTY_KEY, OWL_EMPTY_KEY, hi, lo);
+      if ((o.x == OWL_EMPTY_KEY && o.y == OWL_EMPTY_KEY) || (o.x == hi && o.y == lo)) {
+        if (o.x == OWL_EMPTY_KEY) atomicAdd(&s.cf_fill[tbl], 1u);
+        atomicAdd(&s.cf_cnt[tbl][h], 1u);
+        return;
+      }
+    }
+    h = (h + 1) & (CFK - 1);
   }
   g_insert(a.tab[tbl], tbl, hi, lo, 1, a.status);
 }
 
-__device__ __forceinline__ uint32_t dir_hash(uint64_t hi, uint64_t pg) {
-  return ((uint32_t)hi * 0x9E3779B1u) ^ ((uint32_t)(hi >> 32) * 0x85EBCA77u) ^ ((uint32_t)pg * 0xC2B2AE3Du) ^
-         ((uint32_t)(pg >> 32) * 0x27D4EB2Fu);
+/* 32-bit mixed hash of a directory key: top DIR_LOG bits = home slot, low FILTER_LOG bits = filter slot */
+__device__ __forceinline__ uint32_t dir_hash(uint64_t hi, uint64_t lo) {
+  uint32_t h = ((uint32_t)hi * 0x9E3779B1u) ^ ((uint32_t)(hi >> 32) * 0x85EBCA77u) ^ ((uint32_t)lo * 0xC2B2AE3Du) ^
+               ((uint32_t)(lo >> 32) * 0x27D4EB2Fu);
+  h ^= h >> 15; /* the keys of one program differ in few low bits (ins, j, window): finish the mixing */
+  h *= 0x2C1B3C6Du;
+  h ^= h >> 13;
+  return h;
 }
+#define DIR_PROBES 4
 
-/* Warp-uniform (every lane passes the same key): claims a page for page key (hi, pg), absent from its
-   directory slots h, h+1, on the key's second sighting while pages last; -1 = none (the chunk goes to
-   the global table).  Lane 0 decides, every lane gets its answer. */
-__device__ __noinline__ int page_alloc(FoldSmem& s, uint64_t hi, uint64_t pg, uint32_t h, int lane) {
-  int res = -1;
-  if (lane == 0 && *(volatile unsigned int*)&s.npages < NPAGE && !*(volatile unsigned int*)&s.pages_off) {
-    const uint32_t fp = dir_hash(hi, pg);
-    volatile uint32_t* f = &s.filter[fp & (FILTER_CAP - 1)];
-    if (*f != fp) {
-      *f = fp; /* first sighting: remember it, count this chunk globally */
-    } else {
-      for (int probe = 0; probe < 2; ++probe) {
-        const uint32_t hh = (h + probe) & (DIRCAP - 1);
-        const ulonglong2 o = cas128_shared(&s.dir_key[hh], OWL_EMPTY_KEY, OWL_EMPTY_KEY, hi, pg);
-        if (o.x == OWL_EMPTY_KEY && o.y == OWL_EMPTY_KEY) {
-          const unsigned n = atomicAdd(&s.npages, 1u);
-          if (n < NPAGE) {
-            res = (int)n;
-            s.page_dir[n] = (uint16_t)hh;
-          }
-          *(volatile int*)&s.dir_page[hh] = res; /* pages were zeroed at kernel start */
-          break;
-        }
-        if (o.x == hi && o.y == pg) break; /* claimed meanwhile by another warp: its page id may not be
-                                              published yet; this chunk goes global */
+/* Admission of a recurring key into the CTA directory (lane 0): claims the first free slot of h ..
+   h+DIR_PROBES-1 (the slots lookups probe); a window then gets the next free page.  A key already
+   present, or full slots, leave the directory unchanged. */
+__device__ __noinline__ int dir_admit(FoldSmem& s, uint64_t hi, uint64_t lo, uint32_t h, bool window) {
+  for (int probe = 0; probe < DIR_PROBES; ++probe) {
+    const uint32_t hh = (h + probe) & (DIRCAP - 1);
+    const ulonglong2 o = cas128_shared(&s.dir_key[hh], OWL_EMPTY_KEY, OWL_EMPTY_KEY, hi, lo);
+    if (o.x == OWL_EMPTY_KEY && o.y == OWL_EMPTY_KEY) {
+      if (window) {
+        const unsigned n = atomicAdd(&s.npages, 1u);
+        if (n < NPAGE) s.page_dir[n] = (uint16_t)hh;
+        atomicExch(&s.dir_val[hh], n < NPAGE ? (PV_PAGE | n) : PV_NONE); /* pages were zeroed */
       }
+      return 1;
     }
+    if (o.x == hi && o.y == lo) return 2 + probe;
   }
-  return __shfl_sync(FULL, res, 0);
+  return 0;
 }
 
 __device__ __forceinline__ void report(FoldStatus* st, uint32_t seg_index, uint64_t idx, uint32_t code) {
   atomicMin(&st->first_error, ((unsigned long long)seg_index << 40) | (idx << 3) | code);
 }
 
-/* visits[b] += 1 in the walker's map; returns the new visit ordinal j (reading R8) */
-__device__ __forceinline__ uint32_t visits_inc(uint32_t* vk, uint32_t* vc, uint32_t b, int lane, FoldStatus* st) {
+/* visits[b] += 1 in the warp's map; returns the new visit ordinal j (reading R8).  Entries of
+   older generations (earlier traced warps) count as empty. */
+__device__ __forceinline__ uint32_t visits_inc(uint32_t* vk, uint32_t* vc, uint32_t b, uint32_t gen, int lane,
+                                               FoldStatus* st) {
+  const uint32_t key = (gen << 18) | b;
   const uint32_t h = (b * 0x9E3779B1u) >> 25; /* VCAP = 128 */
   for (int w = 0; w < VCAP / 32; ++w) {
     const uint32_t pos = (h + w * 32 + lane) & (VCAP - 1);
     const uint32_t k = vk[pos];
-    const unsigned found = __ballot_sync(FULL, k == b);
-    const unsigned empty = __ballot_sync(FULL, k == 0xFFFFFFFFu);
+    const unsigned found = __ballot_sync(FULL, k == key);
+    const unsigned empty = __ballot_sync(FULL, (k >> 18) != gen);
     if (found | empty) {
       const bool hit = found && (!empty || __ffs(found) < __ffs(empty));
       const uint32_t p = (h + w * 32 + __ffs(hit ? found : empty) - 1) & (VCAP - 1);
@@ -262,7 +273,7 @@ __device__ __forceinline__ uint32_t visits_inc(uint32_t* vk, uint32_t* vc, uint3
           j = vc[p] + 1;
           vc[p] = j;
         } else {
-          vk[p] = b;
+          vk[p] = key;
           vc[p] = 1;
         }
       }
@@ -294,31 +305,61 @@ __device__ __forceinline__ uint64_t first_warp_start(const uint4* rec, uint64_t 
   return hi;
 }
 
-enum { W_ACTIVE = 1u, W_INWARP = 2u, W_SKIP = 4u };
+/* Admissions of the keys whose sightings reached ADMIT (rare): one distinct key at a time, by lane 0. */
+__device__ __noinline__ void admit_ready(FoldSmem& s, bool ready, uint64_t hi, uint64_t lo, uint32_t h0, uint32_t fi,
+                                         bool window, int lane) {
+  unsigned rm = __ballot_sync(FULL, ready);
+  while (rm) {
+    const int L = __ffs(rm) - 1;
+    const uint64_t ah = __shfl_sync(FULL, hi, L), al = __shfl_sync(FULL, lo, L);
+    const uint32_t ahh = __shfl_sync(FULL, h0, L), afi = __shfl_sync(FULL, fi, L);
+    if (lane == 0) {
+      dir_admit(s, ah, al, ahh, window);
+      s.filt[afi] = 0;
+    }
+    rm &= ~__ballot_sync(FULL, hi == ah && lo == al);
+  }
+}
 
-/* Per-walker state in registers (warp-uniform). */
+enum { W_INWARP = 2u, W_SKIP = 4u };
+
+/* Per-warp walk state in registers (warp-uniform). */
 struct Walker {
-  const uint4* p;   /* next record */
-  uint64_t khi;     /* slot<<48 | cur<<30 | curj: the address key of the current context (ins added per lane) */
+  const uint4* p; /* next record */
+  uint64_t khi;   /* slot<<48 | cur<<30 | curj: address key of the current context (ins added per chunk) */
   uint32_t g0, cur;
+  uint32_t want;  /* meta of a fast-path record modulo lane and ins: MEM | cur<<8 (impossible when skipping) */
   uint32_t st;
+  uint32_t gen;   /* visit-map generation of the traced warp */
 };
 
 /* Slow path of one chunk (BB entries, warp end, malformed records): applies the BB entries, computes the
-   key of every good MEM lane, advances the walker.  Mirrors the oracle walk. */
-__device__ __forceinline__ void slow_chunk(const uint4 r, const unsigned vm, Walker& w, RunDesc& d,
+   key of every good MEM lane, advances the walker past the last BB_ENTRY (or the valid records) and
+   returns the number of records consumed.  Mirrors the oracle walk. */
+struct SlowRes {
+  Walker w;
+  uint64_t khi, lo; /* key of this lane's record if good */
+  int nproc;        /* records consumed */
+  int good;
+};
+
+/* noinline (and everything by value): the slow path is rare, and keeping it out of the unrolled fast
+   loop keeps the kernel within the instruction cache */
+__device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Walker w, RunDesc& d,
                                            const FoldArgs& a, FoldSmem& s, uint32_t* vk, uint32_t* vc,
-                                           const int lane, bool& good, uint64_t& khi_out, uint64_t& lo_out) {
+                                           const int lane) {
+  bool good;
+  uint64_t khi_out, lo_out;
   const int nvalid = vm == FULL ? 32 : __ffs(~vm) - 1;
   const bool active = lane < nvalid;
-  int nproc = nvalid; /* records consumed: up to the last BB_ENTRY, so the next chunk starts on an
-                         instruction boundary (one attribute per fast chunk) */
+  int nproc = nvalid;
   const uint64_t idx = (uint64_t)(w.p - d.rec) + lane;
   const uint64_t addr = (uint64_t)r.x | ((uint64_t)r.y << 32);
   const uint32_t meta = r.w;
   const uint32_t bbf = (meta >> 8) & 0x3FFFFu;
   const uint32_t ins = meta & 0xFFu;
   good = false;
+  khi_out = lo_out = 0;
   if (!(w.st & W_SKIP)) {
     const bool isbb = active && (meta >> 31) == 0;
     const bool bbbad = isbb && (addr != 0 || (meta & 0x7C0000FFu) != 0);
@@ -334,21 +375,20 @@ __device__ __forceinline__ void slow_chunk(const uint4 r, const unsigned vm, Wal
         const int k = __ffs(m) - 1;
         m &= m - 1;
         const uint32_t b = __shfl_sync(FULL, bbf, k);
-        if (a.mode == 0 && lane == 0) {
-          if (w.cur == OWL_NONE_BB) {
-            cf_insert(s, a, T_EDGE, slot_hi | OWL_SENTINEL, b); /* S -> first BB */
-          } else {
-            cf_insert(s, a, T_EDGE, slot_hi | w.cur, b);       /* cur -> b */
+        if (a.mode == 0 && lane < 3) { /* node, edge, triple cell of this entry: one lane (and table) each */
+          if (lane == T_NODE) cf_insert(s, a, T_NODE, slot_hi | b, 0);
+          else if (lane == T_EDGE) /* S -> first BB, else cur -> b */
+            cf_insert(s, a, T_EDGE, slot_hi | (w.cur == OWL_NONE_BB ? OWL_SENTINEL : w.cur), b);
+          else if (w.cur != OWL_NONE_BB)
             cf_insert(s, a, T_TRIPLE, slot_hi | w.cur, ((uint64_t)prev << 32) | b);
-          }
-          cf_insert(s, a, T_NODE, slot_hi | b, 0);
         }
         if (w.cur != OWL_NONE_BB) prev = w.cur;
         w.cur = b;
-        curj = visits_inc(vk, vc, b, lane, a.status);
+        curj = visits_inc(vk, vc, b, w.gen, lane, a.status);
         if (lane == k) myj = curj;
       }
       w.khi = ((uint64_t)d.slot << 48) | ((uint64_t)w.cur << 30) | (uint64_t)curj;
+      w.want = 0x80000000u | (w.cur << 8);
       if (curj > OWL_MAX_J && lane == 0) atomicOr(&a.status->limit, 1u);
       __syncwarp();
       if (lane == 0) {
@@ -356,8 +396,8 @@ __device__ __forceinline__ void slow_chunk(const uint4 r, const unsigned vm, Wal
         d.curj = curj;
       }
       __syncwarp();
+      nproc = 32 - __clz(bbmask); /* consume up to the last BB_ENTRY: the next chunk starts aligned */
     }
-    if (bbmask) nproc = 32 - __clz(bbmask);
     const bool ismem = lane < nproc && (meta >> 31) != 0;
     const unsigned lt = bbmask & ((1u << lane) - 1u);
     const int L = lt ? 31 - __clz(lt) : lane;
@@ -381,18 +421,26 @@ __device__ __forceinline__ void slow_chunk(const uint4 r, const unsigned vm, Wal
   }
   w.p += nproc;
   if (nvalid < 32 && nproc == nvalid) { /* warp end: last BB -> S */
-    if (a.mode == 0 && !(w.st & W_SKIP) && w.cur != OWL_NONE_BB && lane == 0) {
-      cf_insert(s, a, T_EDGE, ((uint64_t)d.slot << 32) | w.cur, OWL_SENTINEL);
-      cf_insert(s, a, T_TRIPLE, ((uint64_t)d.slot << 32) | w.cur, ((uint64_t)d.prev << 32) | OWL_SENTINEL);
+    if (a.mode == 0 && !(w.st & W_SKIP) && w.cur != OWL_NONE_BB && (lane == T_EDGE || lane == T_TRIPLE)) {
+      const uint64_t hi = ((uint64_t)d.slot << 32) | w.cur;
+      if (lane == T_EDGE) cf_insert(s, a, T_EDGE, hi, OWL_SENTINEL);
+      else cf_insert(s, a, T_TRIPLE, hi, ((uint64_t)d.prev << 32) | OWL_SENTINEL);
     }
     w.st &= ~W_INWARP;
   }
+  SlowRes res;
+  res.w = w;
+  res.khi = khi_out;
+  res.lo = lo_out;
+  res.nproc = nproc;
+  res.good = good;
+  return res;
 }
 
 __device__ __forceinline__ void begin_traced_warp(Walker& w, RunDesc& d, const FoldArgs& a, uint32_t* vk,
                                                   int lane) {
   w.g0 = __ldg(&w.p->z);
-  w.st = (w.st & ~W_SKIP) | W_INWARP;
+  w.st = W_INWARP;
   if (w.g0 >= d.n_warps) { /* every record of this warp is malformed (the first one is reported) */
     if (lane == 0) report(a.status, d.seg_index, (uint64_t)(w.p - d.rec), KERR_GWARP);
     w.st |= W_SKIP;
@@ -401,7 +449,10 @@ __device__ __forceinline__ void begin_traced_warp(Walker& w, RunDesc& d, const F
     if (atomicOr(&d.seen[w.g0 >> 5], bit) & bit)
       atomicMin(&a.status->not_warp_major, ((unsigned long long)d.seg_index << 32) | w.g0);
   }
-  for (int i = lane; i < VCAP; i += 32) vk[i] = 0xFFFFFFFFu;
+  if (++w.gen > VGEN_MAX) { /* generations wrapped: clear the map */
+    for (int i = lane; i < VCAP; i += 32) vk[i] = 0;
+    w.gen = 1;
+  }
   if (lane == 0) {
     d.prev = OWL_SENTINEL;
     d.curj = 0;
@@ -409,6 +460,7 @@ __device__ __forceinline__ void begin_traced_warp(Walker& w, RunDesc& d, const F
   __syncwarp();
   w.cur = OWL_NONE_BB;
   w.khi = 0;
+  w.want = 1u; /* no record matches until the first BB_ENTRY (and never while skipping) */
 }
 
 __device__ __forceinline__ const FoldGroup& group_of(const FoldArgs& a, unsigned long long item) {
@@ -420,6 +472,22 @@ __device__ __forceinline__ const FoldGroup& group_of(const FoldArgs& a, unsigned
   return a.groups[lo];
 }
 
+/* lane i of the result = record (i + k) of the 64-record window (lo, hi), 0 < k < 32 */
+__device__ __forceinline__ uint4 funnel(const uint4 lo, const uint4 hi, int k, int lane) {
+  const int src = (lane + k) & 31;
+  const bool from_lo = lane + k < 32;
+  uint4 r;
+  const uint32_t ax = __shfl_sync(FULL, lo.x, src), bx = __shfl_sync(FULL, hi.x, src);
+  const uint32_t ay = __shfl_sync(FULL, lo.y, src), by = __shfl_sync(FULL, hi.y, src);
+  const uint32_t az = __shfl_sync(FULL, lo.z, src), bz = __shfl_sync(FULL, hi.z, src);
+  const uint32_t aw = __shfl_sync(FULL, lo.w, src), bw = __shfl_sync(FULL, hi.w, src);
+  r.x = from_lo ? ax : bx;
+  r.y = from_lo ? ay : by;
+  r.z = from_lo ? az : bz;
+  r.w = from_lo ? aw : bw;
+  return r;
+}
+
 __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs args) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   FoldSmem& s = *reinterpret_cast<FoldSmem*>(smem_raw);
@@ -427,32 +495,36 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   if (threadIdx.x == 0) {
     a = args;
-    s.cf_fill = 0;
     s.npages = 0;
-    s.pages_off = args.mode == 8 ? 1u : 0u; /* experiment mode 8: global table only */
-    s.page_total = 0;
+    s.off = args.mode == 8 ? 1u : 0u; /* experiment mode 8: global table only */
+    s.walked = 0;
   }
-  for (int i = threadIdx.x; i < CF_CAP; i += FOLD_THREADS) {
-    s.cf_key[i] = make_ulonglong2(OWL_EMPTY_KEY, OWL_EMPTY_KEY);
-    s.cf_cnt[i] = 0;
+  if (threadIdx.x < 3) s.cf_fill[threadIdx.x] = 0;
+  for (int i = threadIdx.x; i < 3 * CFK; i += FOLD_THREADS) {
+    (&s.cf_key[0][0])[i] = make_ulonglong2(OWL_EMPTY_KEY, OWL_EMPTY_KEY);
+    (&s.cf_cnt[0][0])[i] = 0;
   }
-  for (int i = threadIdx.x; i < NPAGE * PAGE_BINS; i += FOLD_THREADS) (&s.page[0][0])[i] = 0;
+  for (int i = threadIdx.x; i < NPAGE * PAGE_BINS / 4; i += FOLD_THREADS)
+    reinterpret_cast<uint4*>(&s.page[0][0])[i] = make_uint4(0, 0, 0, 0);
   for (int i = threadIdx.x; i < DIRCAP; i += FOLD_THREADS) {
     s.dir_key[i] = make_ulonglong2(OWL_EMPTY_KEY, OWL_EMPTY_KEY);
-    s.dir_page[i] = -1;
+    s.dir_val[i] = 0;
   }
-  for (int i = threadIdx.x; i < FILTER_CAP; i += FOLD_THREADS) s.filter[i] = 0;
+  uint32_t* vk = s.vkey[warp];
+  uint32_t* vc = s.vcnt[warp];
+  for (int i = lane; i < VCAP; i += 32) vk[i] = 0;
+  for (int i = threadIdx.x; i < (1 << FILTER_LOG); i += FOLD_THREADS) s.filt[i] = 0;
   __syncthreads();
   const uint64_t pol = evict_first_policy();
   const uint64_t tile = 1ull << a.tile_shift;
   const DevTable tab = a.tab[T_ADDR];
   const uint32_t shift = tab_shift(tab.cap);
-  RunDesc& d = s.rd[warp][0];
-  uint32_t* vk = s.vkey[warp][0];
-  uint32_t* vc = s.vcnt[warp][0];
+  RunDesc& d = s.rd[warp];
   uint32_t claims = 0;
-  unsigned long long ptot = 0; /* this warp's page adds since the last item end */
-  uint32_t padds = 0;          /* lane-adds served by pages (statistics) */
+  uint32_t gen = 0;
+#ifdef OWL_FOLD_STATS
+  unsigned long long stat[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#endif
 
   for (;;) {
     unsigned long long item = 0;
@@ -469,23 +541,23 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     const uint64_t e = b + tile < sg.n ? b + tile : sg.n;
     if (lane == 0) {
       d.rec = sg.rec;
-      d.end = sg.rec + sg.n;
-      d.tile_end = sg.rec + e;
       d.seen = sg.seen;
       d.slot = sg.slot;
       d.n_warps = sg.n_warps;
       d.seg_index = sg.seg_index;
     }
     const uint4* const end = sg.rec + sg.n;
-#ifdef OWL_DEBUG_CHECKS
-    if (b > sg.n || e > sg.n) { printf("bad tile b %llu e %llu n %llu\n", (unsigned long long)b, (unsigned long long)e, (unsigned long long)sg.n); __trap(); }
-#endif
     const uint4* const tile_end = sg.rec + e;
     Walker w;
     w.p = sg.rec + first_warp_start(sg.rec, b, e, lane);
-    w.st = W_ACTIVE;
+    const uint4* p_acc = w.p; /* records walked since the last accounting */
+    w.st = 0;
     w.g0 = w.cur = 0;
     w.khi = 0;
+    w.want = 1u;
+    w.gen = gen;
+    /* shared counting stays open while the CTA's walked records cannot wrap a 32-bit counter */
+    bool shared_on = !*(volatile unsigned int*)&s.off;
     if (lane < PF_DIST && a.mode != 3) { /* prime the L2 prefetch window */
       const char* q = (const char*)(((((uintptr_t)w.p) >> PF_LOG) + lane) << PF_LOG);
       if (q < (const char*)end) {
@@ -500,12 +572,25 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         if (w.p >= tile_end) break;
         begin_traced_warp(w, d, a, vk, lane);
       }
-      /* FOLD_U chunks of 32 records: one 128-bit load per lane per chunk */
+      if ((uint64_t)(w.p - p_acc) > (1ull << 22)) { /* very long traced warp: account as we go */
+        if (lane == 0) {
+          const unsigned long long n = (unsigned long long)(w.p - p_acc);
+          if (atomicAdd(&s.walked, n) + n > SHARED_TOTAL_LIMIT) s.off = 1;
+        }
+        __syncwarp();
+        p_acc = w.p;
+        shared_on = !*(volatile unsigned int*)&s.off;
+      }
       uint4 rr[FOLD_U];
+      if (w.p + 32 * FOLD_U <= end) {
 #pragma unroll
-      for (int u = 0; u < FOLD_U; ++u) {
-        const uint4* q = w.p + u * 32 + lane;
-        rr[u] = q < end ? ld_stream(q, pol) : make_uint4(0, 0, 0xFFFFFFFFu, 0);
+        for (int u = 0; u < FOLD_U; ++u) rr[u] = ld_stream(w.p + u * 32 + lane, pol);
+      } else {
+#pragma unroll
+        for (int u = 0; u < FOLD_U; ++u) {
+          const uint4* q = w.p + u * 32 + lane;
+          rr[u] = q < end ? ld_stream(q, pol) : make_uint4(0, 0, 0xFFFFFFFFu, 0);
+        }
       }
       if (a.mode != 3) { /* keep PF_DIST granules of the stream in flight to L2 */
         const uintptr_t g1 = ((uintptr_t)(w.p + 32 * FOLD_U)) >> PF_LOG;
@@ -517,110 +602,119 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
           }
         }
       }
-      /* fast path: every record of the U chunks is a well-formed MEM record of the current BB */
-      const uint32_t want = 0x80000000u | (w.cur << 8);
-      bool ok = !(w.st & W_SKIP) && (w.p + 32 * FOLD_U <= end);
-#pragma unroll
-      for (int u = 0; u < FOLD_U; ++u)
-        ok = ok && rr[u].z == w.g0 && (rr[u].w & 0x83FFFF00u) == want && rr[u].y < 0x90000000u;
-      bool good[FOLD_U], fastc[FOLD_U];
-      uint64_t khi[FOLD_U], klo[FOLD_U];
-      if (__all_sync(FULL, ok)) {
-#pragma unroll
-        for (int u = 0; u < FOLD_U; ++u) {
-          good[u] = fastc[u] = true;
-          khi[u] = w.khi | ((uint64_t)(rr[u].w & 0xFFu) << 22);
-          klo[u] = (uint64_t)rr[u].x | ((uint64_t)rr[u].y << 32);
-        }
-        w.p += 32 * FOLD_U;
-      } else {
-        bool live = true; /* false once the traced warp ended inside this batch: later chunks are reloaded */
-#pragma unroll
-        for (int u = 0; u < FOLD_U; ++u) {
-          good[u] = fastc[u] = false;
-          khi[u] = klo[u] = 0;
-          if (!live) continue;
-          const bool valid = (w.p + lane < end) && rr[u].z == w.g0;
-          const bool fast_ok = valid && (rr[u].w & 0x83FFFF00u) == want && rr[u].y < 0x90000000u;
-          if (__all_sync(FULL, fast_ok) && !(w.st & W_SKIP)) {
-            good[u] = fastc[u] = true;
-            khi[u] = w.khi | ((uint64_t)(rr[u].w & 0xFFu) << 22);
-            klo[u] = (uint64_t)rr[u].x | ((uint64_t)rr[u].y << 32);
-            w.p += 32;
-          } else {
-            const uint4* p0 = w.p;
-            slow_chunk(rr[u], __ballot_sync(FULL, valid), w, d, a, s, vk, vc, lane, good[u], khi[u], klo[u]);
-            live = (w.st & W_INWARP) != 0 && w.p == p0 + 32; /* else later chunks are reloaded */
-          }
-        }
-      }
-      if (a.mode != 0 && a.mode < 5) continue; /* experiment modes: 5 probe only, 6 RED only, 7 no RED */
-
-      /* A3, "merge identical thread traces" before any atomic:
-         - a fast chunk whose 32 keys are equal (broadcast access) is one add of 32;
-         - otherwise the chunk (one attribute after realignment) looks its page key up in the CTA's
-           page directory (branch-free 2-slot probe, same address for every lane: a broadcast read) and
-           the lanes of that page add into shared-memory bins; a missing page is allocated on the key's
-           second sighting (lane 0, rare);
-         - what is left (slow chunks, pages exhausted, wide-range or unaligned addresses) goes to the
-           global table: first probes of all chunks in flight together, predicated REDs, rare misses. */
       bool lead[FOLD_U];
       uint32_t cnt[FOLD_U];
+      uint64_t khi[FOLD_U], klo[FOLD_U];
       unsigned any_lead = 0;
+      bool stop = false; /* the traced warp ended inside the step: the rest is reloaded */
 #pragma unroll
       for (int u = 0; u < FOLD_U; ++u) {
-        lead[u] = good[u];
+        lead[u] = false;
         cnt[u] = 1;
-        if (fastc[u]) { /* the key's upper word is warp-uniform on a fast chunk */
-          const uint32_t x0l = __shfl_sync(FULL, (uint32_t)klo[u], 0);
-          const uint32_t x0h = __shfl_sync(FULL, (uint32_t)(klo[u] >> 32), 0);
-          const uint32_t h0l = __shfl_sync(FULL, (uint32_t)khi[u], 0);
-          const bool eq_ins = (uint32_t)khi[u] == h0l;
-          if (__all_sync(FULL, eq_ins && (uint32_t)klo[u] == x0l && (uint32_t)(klo[u] >> 32) == x0h)) {
+        if (stop) continue;
+        const uint4 r = rr[u];
+        /* fast path: a well-formed MEM record of the current BB of this traced warp */
+        const bool ok = r.z == w.g0 && (r.w & 0x83FFFF00u) == w.want && r.y < 0x90000000u;
+        if (__all_sync(FULL, ok)) {
+          STAT(0);
+          w.p += 32;
+          khi[u] = w.khi | ((uint64_t)(r.w & 0xFFu) << 22);
+          klo[u] = ((uint64_t)r.y << 32) | r.x;
+          lead[u] = true;
+          if (a.mode == 2) { /* experiment: stream + walk only */
+            lead[u] = false;
+            continue;
+          }
+          const uint32_t m0 = __shfl_sync(FULL, r.w, 0);
+          const uint32_t x0l = __shfl_sync(FULL, r.x, 0), x0h = __shfl_sync(FULL, r.y, 0);
+          const bool bc = __all_sync(FULL, ((r.w ^ m0) & 0xFFu) == 0 && r.x == x0l && r.y == x0h);
+          if (bc) { /* broadcast: one cell, 32 adds (lane 0) */
             lead[u] = lane == 0;
             cnt[u] = 32;
-          } else if (!*(volatile unsigned int*)&s.pages_off) {
-            const uint64_t Kh = (khi[u] & 0xFFFFFFFF00000000ull) | h0l;
-            const uint64_t Kp = (((uint64_t)x0h << 32) | x0l) >> 10;
-            const bool mine = eq_ins && (klo[u] >> 10) == Kp && (klo[u] & 3u) == 0;
-            const uint32_t h = dir_hash(Kh, Kp) >> (32 - DIR_LOG);
-            const ulonglong2 k0 = s.dir_key[h], k1 = s.dir_key[(h + 1) & (DIRCAP - 1)];
-            const bool f0 = k0.x == Kh && k0.y == Kp, f1 = k1.x == Kh && k1.y == Kp;
-            int pid = f0 ? s.dir_page[h] : (f1 ? s.dir_page[(h + 1) & (DIRCAP - 1)] : -1);
-            if (__any_sync(FULL, !f0 && !f1 && (k0.x == OWL_EMPTY_KEY || k1.x == OWL_EMPTY_KEY)))
-              pid = page_alloc(s, Kh, Kp, h, lane);
-            if (pid >= 0 && mine) {
-              atomicAdd(&s.page[pid][(klo[u] >> 2) & (PAGE_BINS - 1)], 1u);
-              ++ptot;
-              ++padds;
-              lead[u] = false;
+          }
+          if (shared_on) {
+            /* per lane: the CTA directory holds (attribute, x) of hot broadcast cells and
+               (attribute, x>>10) of hot 1 KB windows, each window owning a page of keyless 4-byte bins.
+               Every lane decides for itself (no vote): a lane that misses goes to the global table. */
+            const uint64_t lo = bc ? klo[u] : ((klo[u] >> 10) | PAGE_TAG);
+            const uint32_t mh = dir_hash(khi[u], lo);
+            const uint32_t h0 = mh >> (32 - DIR_LOG);
+            uint32_t h = h0;
+            ulonglong2 k = s.dir_key[h];
+            bool f = k.x == khi[u] && k.y == lo;
+            for (int probe = 1; probe < DIR_PROBES && !f && k.x != OWL_EMPTY_KEY; ++probe) {
+              h = (h0 + probe) & (DIRCAP - 1);
+              k = s.dir_key[h];
+              f = k.x == khi[u] && k.y == lo;
             }
+            if (f) {
+              if (bc) {
+                if (lane == 0) atomicAdd(&s.dir_val[h], 32u);
+                lead[u] = false;
+              } else {
+                const uint32_t v = s.dir_val[h];
+                if ((v & PV_PAGE) && (r.x & 3u) == 0) {
+                  atomicAdd(&s.page[v & 0xFFFFu][(r.x >> 2) & (PAGE_BINS - 1)], 1u);
+                  lead[u] = false;
+                  STAT(6);
+                }
+              }
+            }
+            /* a key not in the directory: count a sighting, admit recurring keys */
+            bool ready = false;
+            uint32_t fi = 0;
+            if (!f && (!bc || lane == 0)) {
+              STAT(2);
+              /* 4-way filter bucket: the key's entry, else the entry with the fewest sightings is replaced
+                 (hot keys sharing a bucket do not evict each other); racy updates: counts are approximate */
+              const uint32_t tag = mh & 0xFFFFFF00u;
+              const uint32_t bi = mh & ((1u << (FILTER_LOG - 2)) - 1);
+              const uint4 bk = reinterpret_cast<const uint4*>(s.filt)[bi];
+              const uint32_t e0 = bk.x, e1 = bk.y, e2 = bk.z, e3 = bk.w;
+              uint32_t way, ne;
+              if ((e0 & 0xFFFFFF00u) == tag) { way = 0; ne = e0 + 1; }
+              else if ((e1 & 0xFFFFFF00u) == tag) { way = 1; ne = e1 + 1; }
+              else if ((e2 & 0xFFFFFF00u) == tag) { way = 2; ne = e2 + 1; }
+              else if ((e3 & 0xFFFFFF00u) == tag) { way = 3; ne = e3 + 1; }
+              else {
+                const uint32_t c01 = min(e0 & 0xFFu, e1 & 0xFFu), c23 = min(e2 & 0xFFu, e3 & 0xFFu);
+                way = c01 <= c23 ? ((e0 & 0xFFu) <= (e1 & 0xFFu) ? 0u : 1u) : ((e2 & 0xFFu) <= (e3 & 0xFFu) ? 2u : 3u);
+                ne = tag | 1u;
+              }
+              fi = bi * 4 + way;
+              s.filt[fi] = ne;
+              ready = (ne & 0xFFu) >= ADMIT;
+            }
+            if (__any_sync(FULL, ready)) admit_ready(s, ready, khi[u], lo, h0, fi, !bc, lane);
+          }
+        } else {
+          STAT(1);
+          const SlowRes sr = slow_chunk(r, __ballot_sync(FULL, r.z == w.g0 && w.p + lane < end), w, d, a, s, vk, vc,
+                                        lane);
+          w = sr.w;
+          lead[u] = sr.good;
+          khi[u] = sr.khi;
+          klo[u] = sr.lo;
+          const int k = sr.nproc;
+          if (!(w.st & W_INWARP)) {
+            stop = true;
+          } else if (k < 32) {
+            /* realign the rest of the step to the record after the consumed ones (no reload) */
+#pragma unroll
+            for (int c = FOLD_U - 1; c > u; --c) rr[c] = funnel(rr[c - 1], rr[c], k, lane);
           }
         }
         any_lead |= __ballot_sync(FULL, lead[u]);
+
       }
-      if (!any_lead) continue;
+      if (!any_lead || a.mode == 1) continue;
+      /* global table: first probes of all chunks in flight together, predicated REDs, rare misses */
       uint32_t home[FOLD_U];
       ulonglong4 kk[FOLD_U];
 #pragma unroll
       for (int u = 0; u < FOLD_U; ++u) {
         home[u] = tab_index(khi[u], klo[u], shift);
-#ifdef OWL_DEBUG_CHECKS
-        if (lead[u] && home[u] >= tab.cap) { printf("bad home %u cap %llu shift %u\n", home[u], (unsigned long long)tab.cap, shift); __trap(); }
-#endif
-        kk[u] = ld_bucket_keys_if(lead[u] && a.mode != 6, tab.b + (home[u] >> 1));
-      }
-      if (a.mode == 5) { /* experiment: probe loads only */
-        unsigned sink = 0;
-#pragma unroll
-        for (int u = 0; u < FOLD_U; ++u) sink |= (unsigned)(kk[u].x == khi[u]);
-        if (__all_sync(FULL, sink == 7u)) claims += 1;
-        continue;
-      }
-      if (a.mode == 6) { /* experiment: REDs to the home cells only (counts are wrong) */
-#pragma unroll
-        for (int u = 0; u < FOLD_U; ++u) red_add_if(lead[u], &tab.b[home[u] >> 1].count[0], cnt[u]);
-        continue;
+        kk[u] = ld_bucket_keys_if(lead[u], tab.b + (home[u] >> 1));
       }
       unsigned miss_any = 0;
 #pragma unroll
@@ -628,21 +722,21 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         const bool h0 = kk[u].x == khi[u] && kk[u].y == klo[u];
         const bool h1 = kk[u].z == khi[u] && kk[u].w == klo[u];
         const bool hit = lead[u] && (h0 || h1);
-        red_add_if(hit && a.mode != 7, &tab.b[home[u] >> 1].count[h1 ? 1 : 0], cnt[u]);
+        red_add_if(hit, &tab.b[home[u] >> 1].count[h1 ? 1 : 0], cnt[u]);
         lead[u] = lead[u] && !hit; /* now: missed (absent, or displaced past the home bucket) */
         miss_any |= __ballot_sync(FULL, lead[u]);
       }
       if (miss_any) {
 #pragma unroll
         for (int u = 0; u < FOLD_U; ++u)
-          if (lead[u]) claims += addr_insert_slow(tab, shift, home[u], khi[u], klo[u], cnt[u], a.status);
+          if (lead[u]) claims += addr_insert_slow(tab, home[u], khi[u], klo[u], cnt[u], a.status);
       }
     }
-    if (__any_sync(FULL, ptot != 0)) { /* close the pages before any counter could wrap */
-#pragma unroll
-      for (int o = 16; o; o >>= 1) ptot += __shfl_xor_sync(FULL, ptot, o);
-      if (lane == 0 && atomicAdd(&s.page_total, ptot) + ptot > PAGE_TOTAL_LIMIT) s.pages_off = 1;
-      ptot = 0;
+    gen = w.gen;
+    /* records walked by this item bound every shared counter it touched */
+    if (lane == 0) {
+      const unsigned long long n = (unsigned long long)(w.p - p_acc);
+      if (atomicAdd(&s.walked, n) + n > SHARED_TOTAL_LIMIT) s.off = 1;
     }
     /* cells claimed by this item -> table fill; past the load limit the build stops and regrows */
     if (__any_sync(FULL, claims != 0)) {
@@ -656,10 +750,12 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
       claims = 0;
     }
   }
-#pragma unroll
-  for (int o = 16; o; o >>= 1) padds += __shfl_xor_sync(FULL, padds, o);
-  if (lane == 0) atomicAdd(&a.status->n_bypass, (unsigned long long)padds);
+#ifdef OWL_FOLD_STATS
+  if (lane == 0)
+    for (int i = 0; i < 8; ++i) atomicAdd(&a.status->dbg[i], stat[i]);
+#endif
   __syncthreads();
+  /* flush the CTA's exact partial sums: pages, broadcast cells, CF cells */
   const unsigned np = s.npages < NPAGE ? s.npages : NPAGE;
   if (threadIdx.x == 0) atomicAdd(&a.status->n_flush, (unsigned long long)np);
   for (unsigned i = threadIdx.x; i < np * PAGE_BINS; i += FOLD_THREADS) {
@@ -667,15 +763,18 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     const uint32_t c = s.page[pg][b];
     if (c) {
       const ulonglong2 k = s.dir_key[s.page_dir[pg]];
-      g_insert(tab, T_ADDR, k.x, (k.y << 10) | ((uint64_t)b << 2), c, a.status);
+      g_insert(tab, T_ADDR, k.x, ((k.y & ~PAGE_TAG) << 10) | ((uint64_t)b << 2), c, a.status);
     }
   }
-  for (int i = threadIdx.x; i < CF_CAP; i += FOLD_THREADS) {
-    const ulonglong2 k = s.cf_key[i];
-    if (k.x != OWL_EMPTY_KEY) {
-      const int tbl = (int)(k.x >> 62);
-      g_insert(a.tab[tbl], tbl, k.x & ~(3ull << 62), k.y, s.cf_cnt[i], a.status);
-    }
+  for (int i = threadIdx.x; i < DIRCAP; i += FOLD_THREADS) {
+    const ulonglong2 k = s.dir_key[i];
+    const uint32_t c = s.dir_val[i];
+    if (k.x != OWL_EMPTY_KEY && (k.y & PAGE_TAG) != PAGE_TAG && c) g_insert(tab, T_ADDR, k.x, k.y, c, a.status);
+  }
+  for (int i = threadIdx.x; i < 3 * CFK; i += FOLD_THREADS) {
+    const int tbl = i / CFK;
+    const ulonglong2 k = s.cf_key[tbl][i % CFK];
+    if (k.x != OWL_EMPTY_KEY) g_insert(a.tab[tbl], tbl, k.x, k.y, s.cf_cnt[tbl][i % CFK], a.status);
   }
 }
 

@@ -305,6 +305,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     hs.limit = 0;
     hs.tile_counter = 0;
     hs.n_flush = hs.n_bypass = hs.n_claim = 0;
+    for (int i = 0; i < 8; ++i) hs.dbg[i] = 0;
     cudaMemcpyAsync(ctx->d_status, &hs, sizeof hs, cudaMemcpyHostToDevice, st);
     FoldArgs a;
     a.segs = dsegs;
@@ -316,8 +317,9 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     a.status = ctx->d_status;
     a.mode = getenv("OWL_FOLD_MODE") ? (uint32_t)atoi(getenv("OWL_FOLD_MODE")) : 0u;
     const int per_sm = ctx->cfg.fold_ctas_per_sm ? (int)ctx->cfg.fold_ctas_per_sm : owl_fold_ctas_per_sm();
+    const int grid = ctx->n_sm * per_sm;
     cudaEventRecord(ctx->ev0, st);
-    cudaError_t e = items ? owl_launch_fold(a, ctx->n_sm * per_sm, st) : cudaSuccess;
+    cudaError_t e = items ? owl_launch_fold(a, grid, st) : cudaSuccess;
     cudaEventRecord(ctx->ev1, st);
     if (e == cudaSuccess) e = cudaMemcpyAsync(&hs, ctx->d_status, sizeof hs, cudaMemcpyDeviceToHost, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
@@ -330,8 +332,13 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
       ctx->last_fold_records = nrec;
       ctx->total_fold_ms += ms;
       ctx->total_fold_records += nrec;
-      if (getenv("OWL_FOLD_VERBOSE")) fprintf(stderr, "[owl] fold: %llu records %.3f ms pages %llu page-adds %llu claims %llu\n",
-        (unsigned long long)nrec, ms, hs.n_flush, hs.n_bypass, hs.n_claim);
+      if (getenv("OWL_FOLD_VERBOSE")) {
+        fprintf(stderr, "[owl] fold: %llu records %.3f ms pages %llu page-adds %llu claims %llu\n",
+                (unsigned long long)nrec, ms, hs.n_flush, hs.n_bypass, hs.n_claim);
+        if (hs.dbg[0] | hs.dbg[1])
+          fprintf(stderr, "[owl] fold stats: fast %llu slow %llu dir_miss %llu dir_claim %llu admit %llu bcast %llu page %llu global %llu\n",
+                  hs.dbg[0], hs.dbg[1], hs.dbg[2], hs.dbg[3], hs.dbg[4], hs.dbg[5], hs.dbg[6], hs.dbg[7]);
+      }
     }
   }
   if (status == OWL_OK) {

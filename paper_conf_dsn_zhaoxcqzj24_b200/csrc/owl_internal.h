@@ -63,6 +63,8 @@ struct FoldStatus {
   unsigned long long n_flush;       /* shared-memory pages allocated (all CTAs)                     */
   unsigned long long n_bypass;      /* address lane-adds served by shared-memory pages              */
   unsigned long long n_claim;       /* shared-table cells claimed                                   */
+  unsigned long long dbg[8];        /* OWL_FOLD_STATS builds: fast / slow chunks, directory misses,
+                                       directory claims, page admits, broadcast / page / global chunks */
 };
 
 /* One segment as the fold kernel sees it */
