@@ -11,6 +11,7 @@ Every step of the path runs inside libowl's CUDA kernels; PyTorch only provides 
 from __future__ import annotations
 
 import ctypes
+import weakref
 
 import numpy as np
 
@@ -82,8 +83,10 @@ def _take(ptr, n, dtype):
         if ptr.value:
             L.owl_free(ptr)
         return np.zeros(0, dtype=dtype)
-    out = np.frombuffer(ctypes.string_at(ptr.value, n * dtype.itemsize), dtype=dtype).copy()
-    L.owl_free(ptr)
+    # zero-copy: the array views the library's malloc'd rows and frees them when it is collected
+    buf = (ctypes.c_char * (n * dtype.itemsize)).from_address(ptr.value)
+    out = np.frombuffer(buf, dtype=dtype)
+    weakref.finalize(buf, L.owl_free, ctypes.c_void_p(ptr.value))
     return out
 
 
@@ -141,8 +144,11 @@ class Context:
             self.set_config(**config)
 
     def __del__(self):
-        if getattr(self, "h", None):
-            _lib.load().owl_ctx_destroy(self.h)
+        if getattr(self, "h", None) and _lib is not None:  # modules may be torn down at interpreter exit
+            try:
+                _lib.load().owl_ctx_destroy(self.h)
+            except Exception:  # noqa: BLE001
+                pass
             self.h = None
 
     def set_config(self, addr_capacity=0, cf_capacity=0, max_regrow=0, fold_ctas_per_sm=0, host_chunk_bytes=0):

@@ -42,15 +42,17 @@ using namespace owl_dev;
 
 #define FULL 0xFFFFFFFFu
 #ifndef FOLD_WARPS
-#define FOLD_WARPS 16
+#define FOLD_WARPS 24 /* profiles/r01_v4_ab.txt: U2 W24 beat U1-4 x W16-32 */
 #endif
 #ifndef FOLD_U
-#define FOLD_U 4 /* chunks of 32 records per warp and step */
+#define FOLD_U 2 /* chunks of 32 records per warp and step */
 #endif
 #define FOLD_THREADS (FOLD_WARPS * 32)
 #define CFK 128      /* shared cells per CF table kind (node, edge, triple) */
 #define CFK_LIMIT 96
-#define VCAP 128     /* per-warp visit map (distinct BBs of one traced warp) */
+#ifndef VCAP
+#define VCAP 64     /* per-warp overflow visit map (BBs beyond the 32 held in registers) */
+#endif
 #define VGEN_MAX 0x3FFFu /* visit-map entry = gen<<18 | bb: a new generation per traced warp, 0 = empty */
 #ifndef PF_LOG
 #define PF_LOG 12    /* L2 bulk prefetch granule: 4 KB (256 records) */
@@ -93,7 +95,6 @@ struct RunDesc {
   const uint4* rec; /* segment base */
   uint32_t* seen;
   uint32_t slot, n_warps, seg_index;
-  uint32_t prev, curj;
 };
 
 struct __align__(16) FoldSmem {
@@ -121,9 +122,16 @@ __device__ __forceinline__ uint64_t evict_first_policy() {
 
 __device__ __forceinline__ uint4 ld_stream(const uint4* p, uint64_t pol) {
   uint4 r;
+#ifdef STREAM_NO_HINT
+  (void)pol;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+#else
   asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
                : "l"(p), "l"(pol));
+#endif
   return r;
 }
 
@@ -258,7 +266,7 @@ __device__ __forceinline__ void report(FoldStatus* st, uint32_t seg_index, uint6
 __device__ __forceinline__ uint32_t visits_inc(uint32_t* vk, uint32_t* vc, uint32_t b, uint32_t gen, int lane,
                                                FoldStatus* st) {
   const uint32_t key = (gen << 18) | b;
-  const uint32_t h = (b * 0x9E3779B1u) >> 25; /* VCAP = 128 */
+  const uint32_t h = (b * 0x9E3779B1u) >> (32 - __ffs(VCAP) + 1); /* top log2(VCAP) bits */
   for (int w = 0; w < VCAP / 32; ++w) {
     const uint32_t pos = (h + w * 32 + lane) & (VCAP - 1);
     const uint32_t k = vk[pos];
@@ -323,19 +331,39 @@ __device__ __noinline__ void admit_ready(FoldSmem& s, bool ready, uint64_t hi, u
 
 enum { W_INWARP = 2u, W_SKIP = 4u };
 
-/* Per-warp walk state in registers (warp-uniform). */
+/* Per-warp walk state in registers (warp-uniform except vb / vn). */
 struct Walker {
-  const uint4* p; /* next record */
-  uint64_t khi;   /* slot<<48 | cur<<30 | curj: address key of the current context (ins added per chunk) */
-  uint32_t g0, cur;
-  uint32_t want;  /* meta of a fast-path record modulo lane and ins: MEM | cur<<8 (impossible when skipping) */
+  const uint4* p;  /* next record */
+  uint64_t khi;    /* slot<<48 | cur<<30 | curj: address key of the current context (ins added per chunk) */
+  uint32_t g0, cur, prev, curj, slot;
+  uint32_t want;   /* meta of a fast-path record modulo lane and ins: MEM | cur<<8 (impossible when skipping) */
   uint32_t st;
-  uint32_t gen;   /* visit-map generation of the traced warp */
+  uint32_t gen;    /* generation of the traced warp in the shared overflow visit map */
+  uint32_t vb, vn; /* visit map in registers: lane l holds BB vb and its visit count vn (32 BBs / warp) */
 };
 
-/* Slow path of one chunk (BB entries, warp end, malformed records): applies the BB entries, computes the
-   key of every good MEM lane, advances the walker past the last BB_ENTRY (or the valid records) and
-   returns the number of records consumed.  Mirrors the oracle walk. */
+/* visits[b] += 1 for the traced warp; returns the new visit ordinal j (reading R8).  The first
+   32 distinct BBs of a traced warp live in registers (one per lane), further ones in the shared map. */
+__device__ __forceinline__ uint32_t visit(Walker& w, uint32_t* vk, uint32_t* vc, uint32_t b, int lane,
+                                          FoldStatus* st) {
+  const unsigned m = __ballot_sync(FULL, w.vb == b);
+  if (m) {
+    const int L = __ffs(m) - 1;
+    const uint32_t j = __shfl_sync(FULL, w.vn, L) + 1;
+    if (lane == L) w.vn = j;
+    return j;
+  }
+  const unsigned used = __ballot_sync(FULL, w.vb != 0xFFFFFFFFu);
+  if (used != FULL) {
+    if (lane == __ffs(~used) - 1) {
+      w.vb = b;
+      w.vn = 1;
+    }
+    return 1;
+  }
+  return visits_inc(vk, vc, b, w.gen, lane, st);
+}
+
 struct SlowRes {
   Walker w;
   uint64_t khi, lo; /* key of this lane's record if good */
@@ -365,11 +393,11 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
     const bool bbbad = isbb && (addr != 0 || (meta & 0x7C0000FFu) != 0);
     if (bbbad) report(a.status, d.seg_index, idx, KERR_BBFIELDS);
     const unsigned bbmask = __ballot_sync(FULL, isbb && !bbbad);
-    const uint32_t cur0 = w.cur, j0 = d.curj;
+    const uint32_t cur0 = w.cur, j0 = w.curj;
     uint32_t myj = 0;
     if (bbmask) {
-      uint32_t prev = d.prev, curj = j0;
-      const uint64_t slot_hi = (uint64_t)d.slot << 32;
+      uint32_t prev = w.prev, curj = j0;
+      const uint64_t slot_hi = (uint64_t)w.slot << 32;
       unsigned m = bbmask;
       while (m) {
         const int k = __ffs(m) - 1;
@@ -384,18 +412,14 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
         }
         if (w.cur != OWL_NONE_BB) prev = w.cur;
         w.cur = b;
-        curj = visits_inc(vk, vc, b, w.gen, lane, a.status);
+        curj = visit(w, vk, vc, b, lane, a.status);
         if (lane == k) myj = curj;
       }
-      w.khi = ((uint64_t)d.slot << 48) | ((uint64_t)w.cur << 30) | (uint64_t)curj;
+      w.khi = ((uint64_t)w.slot << 48) | ((uint64_t)w.cur << 30) | (uint64_t)curj;
       w.want = 0x80000000u | (w.cur << 8);
       if (curj > OWL_MAX_J && lane == 0) atomicOr(&a.status->limit, 1u);
-      __syncwarp();
-      if (lane == 0) {
-        d.prev = prev;
-        d.curj = curj;
-      }
-      __syncwarp();
+      w.prev = prev;
+      w.curj = curj;
       nproc = 32 - __clz(bbmask); /* consume up to the last BB_ENTRY: the next chunk starts aligned */
     }
     const bool ismem = lane < nproc && (meta >> 31) != 0;
@@ -416,15 +440,15 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
     }
     good = ismem && code == 0;
     if (good && cj > OWL_MAX_J) atomicOr(&a.status->limit, 1u);
-    khi_out = ((uint64_t)d.slot << 48) | ((uint64_t)cbb << 30) | ((uint64_t)ins << 22) | cj;
+    khi_out = ((uint64_t)w.slot << 48) | ((uint64_t)cbb << 30) | ((uint64_t)ins << 22) | cj;
     lo_out = addr;
   }
   w.p += nproc;
   if (nvalid < 32 && nproc == nvalid) { /* warp end: last BB -> S */
     if (a.mode == 0 && !(w.st & W_SKIP) && w.cur != OWL_NONE_BB && (lane == T_EDGE || lane == T_TRIPLE)) {
-      const uint64_t hi = ((uint64_t)d.slot << 32) | w.cur;
+      const uint64_t hi = ((uint64_t)w.slot << 32) | w.cur;
       if (lane == T_EDGE) cf_insert(s, a, T_EDGE, hi, OWL_SENTINEL);
-      else cf_insert(s, a, T_TRIPLE, hi, ((uint64_t)d.prev << 32) | OWL_SENTINEL);
+      else cf_insert(s, a, T_TRIPLE, hi, ((uint64_t)w.prev << 32) | OWL_SENTINEL);
     }
     w.st &= ~W_INWARP;
   }
@@ -453,11 +477,11 @@ __device__ __forceinline__ void begin_traced_warp(Walker& w, RunDesc& d, const F
     for (int i = lane; i < VCAP; i += 32) vk[i] = 0;
     w.gen = 1;
   }
-  if (lane == 0) {
-    d.prev = OWL_SENTINEL;
-    d.curj = 0;
-  }
   __syncwarp();
+  w.prev = OWL_SENTINEL;
+  w.curj = 0;
+  w.vb = 0xFFFFFFFFu;
+  w.vn = 0;
   w.cur = OWL_NONE_BB;
   w.khi = 0;
   w.want = 1u; /* no record matches until the first BB_ENTRY (and never while skipping) */
@@ -556,6 +580,11 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     w.khi = 0;
     w.want = 1u;
     w.gen = gen;
+    w.slot = sg.slot;
+    w.prev = OWL_SENTINEL;
+    w.curj = 0;
+    w.vb = 0xFFFFFFFFu;
+    w.vn = 0;
     /* shared counting stays open while the CTA's walked records cannot wrap a 32-bit counter */
     bool shared_on = !*(volatile unsigned int*)&s.off;
     if (lane < PF_DIST && a.mode != 3) { /* prime the L2 prefetch window */
@@ -687,6 +716,28 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
             }
             if (__any_sync(FULL, ready)) admit_ready(s, ready, khi[u], lo, h0, fi, !bc, lane);
           }
+        } else if (__shfl_sync(FULL, r.z == w.g0 && (r.w & 0xFC0000FFu) == 0 && r.x == 0 && r.y == 0, 0) &&
+                   !(w.st & W_SKIP) && a.mode == 0) {
+          /* the common slow chunk: a well-formed BB_ENTRY in lane 0 (chunks start on instruction
+             boundaries).  Consume it alone, then realign the rest of the step. */
+          STAT(1);
+          const uint32_t b = (__shfl_sync(FULL, r.w, 0) >> 8) & 0x3FFFFu;
+          const uint64_t slot_hi = (uint64_t)w.slot << 32;
+          if (lane < 3) { /* node / edge / triple cell of this entry, one lane (and table) each */
+            const bool first = w.cur == OWL_NONE_BB;
+            const uint64_t hi = slot_hi | (lane == T_NODE ? b : (first ? OWL_SENTINEL : w.cur));
+            const uint64_t lo = lane == T_NODE ? 0 : (lane == T_EDGE ? (uint64_t)b : (((uint64_t)w.prev << 32) | b));
+            if (lane != T_TRIPLE || !first) cf_insert(s, a, lane, hi, lo);
+          }
+          if (w.cur != OWL_NONE_BB) w.prev = w.cur;
+          w.cur = b;
+          w.curj = visit(w, vk, vc, b, lane, a.status);
+          if (w.curj > OWL_MAX_J && lane == 0) atomicOr(&a.status->limit, 1u);
+          w.khi = ((uint64_t)w.slot << 48) | ((uint64_t)b << 30) | (uint64_t)w.curj;
+          w.want = 0x80000000u | (b << 8);
+          w.p += 1;
+#pragma unroll
+          for (int c = FOLD_U - 1; c > u; --c) rr[c] = funnel(rr[c - 1], rr[c], 1, lane);
         } else {
           STAT(1);
           const SlowRes sr = slow_chunk(r, __ballot_sync(FULL, r.z == w.g0 && w.p + lane < end), w, d, a, s, vk, vc,

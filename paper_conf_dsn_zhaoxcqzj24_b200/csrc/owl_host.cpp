@@ -12,6 +12,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <chrono>
 #include <map>
 #include <string>
 #include <tuple>
@@ -400,7 +401,7 @@ owl_status build_tables(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTa
          bucket and the fold's first probe hits (owl_fold.cu) */
       unsigned long long fill = 0;
       cudaMemcpy(&fill, tab[T_ADDR].fill, sizeof fill, cudaMemcpyDeviceToHost);
-      static const int load_shift = getenv("OWL_ADDR_LOAD_SHIFT") ? atoi(getenv("OWL_ADDR_LOAD_SHIFT")) : 4;
+      static const int load_shift = getenv("OWL_ADDR_LOAD_SHIFT") ? atoi(getenv("OWL_ADDR_LOAD_SHIFT")) : 3;
       ctx->cap_hint[T_ADDR] = std::max(ctx->cap_hint[T_ADDR], std::min<uint64_t>(next_pow2(fill << load_shift), 1ull << 28));
       for (int t = 0; t < T_NUM; ++t) ctx->cap_hint[t] = std::max(ctx->cap_hint[t], cap[t]);
       return OWL_OK;
@@ -414,11 +415,9 @@ owl_status build_tables(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTa
 
 owl_status ensure_sorted(owl_adcfg* g) {
   if (g->sorted_ok) return OWL_OK;
-  for (int t = 0; t < T_NUM; ++t) {
-    owl_sorted_free(&g->sorted[t]);
-    cudaError_t e = owl_table_sorted(g->tab[t], &g->sorted[t], g->ctx->stream);
-    if (e != cudaSuccess) return cuda_fail(e, "canonical sort");
-  }
+  for (int t = 0; t < T_NUM; ++t) owl_sorted_free(&g->sorted[t]);
+  cudaError_t e = owl_tables_sorted(g->tab, T_NUM, g->sorted, g->ctx->stream);
+  if (e != cudaSuccess) return cuda_fail(e, "canonical sort");
   g->sorted_ok = true;
   return OWL_OK;
 }
@@ -679,33 +678,25 @@ OWL_API owl_status owl_diff_adcfg(owl_ctx* ctx, const owl_adcfg* a, const owl_ad
   CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
   owl_adcfg* ga = const_cast<owl_adcfg*>(a);
   owl_adcfg* gb = const_cast<owl_adcfg*>(b);
+  static const bool verbose = getenv("OWL_DIFF_VERBOSE") != nullptr;
+  auto now = [] { return std::chrono::steady_clock::now(); };
+  auto t0 = now();
   owl_status s = ensure_sorted(ga);
+  auto t1 = now();
   if (s == OWL_OK) s = ensure_sorted(gb);
+  auto t2 = now();
   if (s != OWL_OK) return s;
-  std::vector<owl_diff> out;
   const uint32_t NA = 0xFFFFFFFFu;
-  for (int t = 0; t < T_NUM; ++t) {
-    std::vector<DiffCell> d;
-    CUDA_TRY(owl_diff_sorted(ga->sorted[t], gb->sorted[t], d, ctx->stream), "diff");
-    for (const DiffCell& c : d) {
-      owl_diff r;
-      uint32_t slot, x1, x2, x3;
-      uint64_t x;
-      unpack(t, c.k, slot, x1, x2, x3, x);
-      r.table = (uint32_t)t;
-      r.slot = slot;
-      r.bb = r.ins = r.j = r.prev = r.next = NA;
-      r._pad = 0;
-      r.x = 0;
-      if (t == T_NODE) r.bb = x1;
-      else if (t == T_EDGE) { r.prev = x1; r.next = x3; }
-      else if (t == T_TRIPLE) { r.bb = x1; r.prev = x2; r.next = x3; }
-      else { r.bb = x1; r.ins = x2; r.j = x3; r.x = x; }
-      r.count_a = c.ca;
-      r.count_b = c.cb;
-      out.push_back(r);
-    }
-  }
+  owl_diff* dev_rows = nullptr;
+  uint64_t nd = 0;
+  const size_t extra = ga->slots.order.size() + gb->slots.order.size();
+  CUDA_TRY(owl_diff_rows(ga->sorted, gb->sorted, T_NUM, &dev_rows, &nd, extra, ctx->stream), "diff");
+  auto t3 = now();
+  if (verbose)
+    fprintf(stderr, "[owl] diff: sort a %.3f ms, sort b %.3f ms, join + rows %.3f ms (%llu rows)\n",
+            std::chrono::duration<double, std::milli>(t1 - t0).count(),
+            std::chrono::duration<double, std::milli>(t2 - t1).count(),
+            std::chrono::duration<double, std::milli>(t3 - t2).count(), (unsigned long long)nd);
   /* slot table: (slot, kernel_id) -> invocation count */
   std::map<std::pair<uint32_t, uint64_t>, uint64_t> sa, sb;
   for (uint32_t sl : ga->slots.order) sa[{sl, ga->slots.kid[sl]}] = ga->slots.count[sl];
@@ -715,7 +706,7 @@ OWL_API owl_status owl_diff_adcfg(owl_ctx* ctx, const owl_adcfg* a, const owl_ad
   for (auto& e : sb) all[e.first].second = e.second;
   for (auto& e : all)
     if (e.second.first != e.second.second) {
-      owl_diff r;
+      owl_diff& r = dev_rows[nd++];
       r.table = OWL_TABLE_SLOT;
       r.slot = e.first.first;
       r.bb = r.ins = r.j = r.prev = r.next = NA;
@@ -723,11 +714,10 @@ OWL_API owl_status owl_diff_adcfg(owl_ctx* ctx, const owl_adcfg* a, const owl_ad
       r.x = e.first.second;
       r.count_a = e.second.first;
       r.count_b = e.second.second;
-      out.push_back(r);
     }
-  *rows = host_copy(out);
-  *n_rows = out.size();
-  return *rows ? OWL_OK : fail(OWL_ERR_OUT_OF_MEMORY, "diff rows");
+  *rows = dev_rows;
+  *n_rows = nd;
+  return OWL_OK;
 }
 
 namespace {

@@ -115,7 +115,7 @@ struct SortedTable {
 
 cudaError_t owl_table_alloc(DevTable* t, uint64_t cap, cudaStream_t st);
 void owl_table_free(DevTable* t);
-cudaError_t owl_table_sorted(const DevTable& t, SortedTable* out, cudaStream_t st);
+cudaError_t owl_tables_sorted(const DevTable* t, int ntab, SortedTable* out, cudaStream_t st);
 void owl_sorted_free(SortedTable* s);
 /* inserts every cell of a sorted table into a hash table (evidence merge of partial builds / absorb) */
 cudaError_t owl_table_insert_sorted(const DevTable& t, int tbl, const Key128* k, const unsigned long long* c,
@@ -127,6 +127,10 @@ struct DiffCell {
 };
 /* full outer join of two sorted tables: the differing cells in canonical order */
 cudaError_t owl_diff_sorted(const SortedTable& a, const SortedTable& b, std::vector<DiffCell>& out, cudaStream_t st);
+
+/* A5 over all tables at once (canonical order), into malloc'd host rows with room for extra_rows more */
+cudaError_t owl_diff_rows(const SortedTable* A, const SortedTable* B, int ntab, owl_diff** rows, uint64_t* n_rows,
+                          size_t extra_rows, cudaStream_t st);
 
 /* stable bucketing of a segment's records by gwarp (channel-order input, reading R17) */
 cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, uint4* out, uint64_t* perm,

@@ -32,10 +32,12 @@ __global__ void clear_kernel(owl_bucket* b, uint64_t nb) {
   }
 }
 
-/* compaction of non-empty cells (order is irrelevant: a sort follows) */
+/* compaction of non-empty cells (order is irrelevant: a sort follows); also the bitwise OR and AND of the
+   live keys (bits that vary across the table: the radix sort needs only those) */
 __global__ void compact_kernel(const owl_bucket* c, uint64_t cap, Key128* k, unsigned long long* cnt,
-                               unsigned long long* n_out) {
+                               unsigned long long* n_out, unsigned long long* masks /* or_hi, or_lo, and_hi, and_lo */) {
   const int lane = threadIdx.x & 31;
+  unsigned long long ohi = 0, olo = 0, ahi = ~0ull, alo = ~0ull;
   for (uint64_t base = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) & ~31ull; base < cap;
        base += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t i = base + lane;
@@ -56,7 +58,54 @@ __global__ void compact_kernel(const owl_bucket* c, uint64_t cap, Key128* k, uns
       k[o].hi = vhi;
       k[o].lo = vlo;
       cnt[o] = vc;
+      ohi |= vhi;
+      olo |= vlo;
+      ahi &= vhi;
+      alo &= vlo;
     }
+  }
+  for (int o = 16; o; o >>= 1) {
+    ohi |= __shfl_xor_sync(0xFFFFFFFFu, ohi, o);
+    olo |= __shfl_xor_sync(0xFFFFFFFFu, olo, o);
+    ahi &= __shfl_xor_sync(0xFFFFFFFFu, ahi, o);
+    alo &= __shfl_xor_sync(0xFFFFFFFFu, alo, o);
+  }
+  if (lane == 0) {
+    atomicOr(&masks[0], ohi);
+    atomicOr(&masks[1], olo);
+    atomicAnd(&masks[2], ahi);
+    atomicAnd(&masks[3], alo);
+  }
+}
+
+/* Order-preserving key compaction for the radix sort: the bits that vary across a table's keys, packed
+   (hi's above lo's, each in significance order) into one u64 — equal constant bits make the packed
+   order the (hi, lo) order.  Runs are (shift, length) of the varying-bit mask, packed from the top. */
+struct PackRuns {
+  int n;
+  unsigned char word[48], shift[48], len[48], pos[48];
+};
+
+__global__ void pack_kernel(const Key128* k, uint64_t n, PackRuns r, unsigned long long* ck, uint32_t* idx) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const Key128 q = k[i];
+    unsigned long long v = 0;
+    for (int t = 0; t < r.n; ++t) {
+      const unsigned long long w = r.word[t] ? q.lo : q.hi;
+      const unsigned long long f = (w >> r.shift[t]) & (r.len[t] == 64 ? ~0ull : ((1ull << r.len[t]) - 1));
+      v |= f << r.pos[t];
+    }
+    ck[i] = v;
+    idx[i] = (uint32_t)i;
+  }
+}
+
+__global__ void gather_sorted_kernel(const Key128* k0, const unsigned long long* c0, const uint32_t* idx, uint64_t n,
+                                     Key128* k, unsigned long long* c) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t j = idx[i];
+    k[i] = k0[j];
+    c[i] = c0[j];
   }
 }
 
@@ -214,30 +263,103 @@ void owl_sorted_free(SortedTable* s) {
   s->n = 0;
 }
 
-cudaError_t owl_table_sorted(const DevTable& t, SortedTable* out, cudaStream_t st) {
-  unsigned long long n = 0;
-  cudaError_t e = cudaMemcpyAsync(&n, t.fill, sizeof n, cudaMemcpyDeviceToHost, st);
+/* varying-bit runs of (hi, lo) masks, packed from bit nb-1 down; false if more than 64 bits vary */
+static bool pack_runs(unsigned long long mhi, unsigned long long mlo, PackRuns* r, int* nb) {
+  const int total = __builtin_popcountll(mhi) + __builtin_popcountll(mlo);
+  if (total > 64) return false;
+  r->n = 0;
+  int top = total;
+  for (int word = 0; word < 2; ++word) {
+    unsigned long long m = word ? mlo : mhi;
+    /* most significant run first */
+    while (m) {
+      const int hb = 63 - __builtin_clzll(m);
+      int lb = hb;
+      while (lb > 0 && ((m >> (lb - 1)) & 1)) --lb;
+      const int len = hb - lb + 1;
+      if (r->n >= 48) return false;
+      top -= len;
+      r->word[r->n] = (unsigned char)word;
+      r->shift[r->n] = (unsigned char)lb;
+      r->len[r->n] = (unsigned char)len;
+      r->pos[r->n] = (unsigned char)top;
+      ++r->n;
+      m &= (len == 64) ? 0ull : ~(((1ull << len) - 1) << lb);
+    }
+  }
+  *nb = total;
+  return true;
+}
+
+/* Canonical order of ntab tables at once (compaction, then a radix sort of the packed varying key bits,
+   or of the full 128-bit keys for small tables); three host synchronisations in all. */
+cudaError_t owl_tables_sorted(const DevTable* t, int ntab, SortedTable* out, cudaStream_t st) {
+  std::vector<unsigned long long> n(ntab, 0);
+  cudaError_t e = cudaSuccess;
+  for (int i = 0; i < ntab && e == cudaSuccess; ++i) e = cudaMemcpyAsync(&n[i], t[i].fill, 8, cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   if (e != cudaSuccess) return e;
-  Key128* k0 = (Key128*)owl_dev_alloc(n * sizeof(Key128));
-  unsigned long long* c0 = (unsigned long long*)owl_dev_alloc(n * sizeof(unsigned long long));
-  out->k = (Key128*)owl_dev_alloc(n * sizeof(Key128));
-  out->c = (unsigned long long*)owl_dev_alloc(n * sizeof(unsigned long long));
-  unsigned long long* dn = (unsigned long long*)owl_dev_alloc(sizeof(unsigned long long));
-  if (!k0 || !c0 || !out->k || !out->c || !dn) {
-    owl_dev_free(k0); owl_dev_free(c0); owl_dev_free(dn); owl_sorted_free(out);
-    return cudaErrorMemoryAllocation;
+  std::vector<void*> scratch;
+  auto alloc = [&](size_t bytes) { void* p = owl_dev_alloc(bytes); scratch.push_back(p); return p; };
+  std::vector<Key128*> k0(ntab);
+  std::vector<unsigned long long*> c0(ntab);
+  unsigned long long* dn = (unsigned long long*)alloc(5 * 8 * ntab);
+  if (!dn) e = cudaErrorMemoryAllocation;
+  std::vector<unsigned long long> init(5 * ntab);
+  for (int i = 0; i < ntab; ++i) {
+    init[5 * i] = init[5 * i + 1] = init[5 * i + 2] = 0;
+    init[5 * i + 3] = init[5 * i + 4] = ~0ull;
   }
-  cudaMemsetAsync(dn, 0, sizeof(unsigned long long), st);
-  compact_kernel<<<grid_for(t.cap, 256), 256, 0, st>>>(t.b, t.cap, k0, c0, dn);
-  size_t tmp = 0;
-  cub::DeviceRadixSort::SortPairs(nullptr, tmp, k0, out->k, c0, out->c, (int64_t)n, KeyDecomp{}, st);
-  void* dt = owl_dev_alloc(tmp);
-  if (!dt) e = cudaErrorMemoryAllocation;
-  else e = cub::DeviceRadixSort::SortPairs(dt, tmp, k0, out->k, c0, out->c, (int64_t)n, KeyDecomp{}, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(dn, init.data(), 5 * 8 * ntab, cudaMemcpyHostToDevice, st);
+  bool any_large = false;
+  for (int i = 0; i < ntab && e == cudaSuccess; ++i) {
+    k0[i] = (Key128*)alloc(n[i] * sizeof(Key128));
+    c0[i] = (unsigned long long*)alloc(n[i] * 8);
+    out[i].k = (Key128*)owl_dev_alloc(n[i] * sizeof(Key128));
+    out[i].c = (unsigned long long*)owl_dev_alloc(n[i] * 8);
+    out[i].n = n[i];
+    if (!k0[i] || !c0[i] || !out[i].k || !out[i].c) { e = cudaErrorMemoryAllocation; break; }
+    compact_kernel<<<grid_for(t[i].cap, 256), 256, 0, st>>>(t[i].b, t[i].cap, k0[i], c0[i], dn + 5 * i, dn + 5 * i + 1);
+    any_large |= n[i] > 4096;
+  }
+  std::vector<unsigned long long> masks(5 * ntab, 0);
+  if (e == cudaSuccess && any_large) {
+    e = cudaMemcpyAsync(masks.data(), dn, 5 * 8 * ntab, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  }
+  for (int i = 0; i < ntab && e == cudaSuccess; ++i) {
+    if (!n[i]) continue;
+    const unsigned long long* m = &masks[5 * i + 1]; /* or_hi, or_lo, and_hi, and_lo */
+    PackRuns runs;
+    int nb = 0;
+    if (n[i] > 4096 && pack_runs(m[0] ^ m[2], m[1] ^ m[3], &runs, &nb)) {
+      /* large table: radix-sort the packed varying bits (a few passes instead of 16) and gather */
+      unsigned long long* ck = (unsigned long long*)alloc(n[i] * 8);
+      unsigned long long* ck2 = (unsigned long long*)alloc(n[i] * 8);
+      uint32_t* ix = (uint32_t*)alloc(n[i] * 4);
+      uint32_t* ix2 = (uint32_t*)alloc(n[i] * 4);
+      if (!ck || !ck2 || !ix || !ix2) { e = cudaErrorMemoryAllocation; break; }
+      pack_kernel<<<grid_for(n[i], 256), 256, 0, st>>>(k0[i], n[i], runs, ck, ix);
+      size_t tmp = 0;
+      const int eb = nb > 0 ? nb : 1;
+      cub::DeviceRadixSort::SortPairs(nullptr, tmp, ck, ck2, ix, ix2, (int64_t)n[i], 0, eb, st);
+      void* dt = alloc(tmp);
+      if (!dt) { e = cudaErrorMemoryAllocation; break; }
+      e = cub::DeviceRadixSort::SortPairs(dt, tmp, ck, ck2, ix, ix2, (int64_t)n[i], 0, eb, st);
+      if (e == cudaSuccess)
+        gather_sorted_kernel<<<grid_for(n[i], 256), 256, 0, st>>>(k0[i], c0[i], ix2, n[i], out[i].k, out[i].c);
+    } else {
+      size_t tmp = 0;
+      cub::DeviceRadixSort::SortPairs(nullptr, tmp, k0[i], out[i].k, c0[i], out[i].c, (int64_t)n[i], KeyDecomp{}, st);
+      void* dt = alloc(tmp);
+      if (!dt) { e = cudaErrorMemoryAllocation; break; }
+      e = cub::DeviceRadixSort::SortPairs(dt, tmp, k0[i], out[i].k, c0[i], out[i].c, (int64_t)n[i], KeyDecomp{}, st);
+    }
+  }
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  owl_dev_free(dt); owl_dev_free(k0); owl_dev_free(c0); owl_dev_free(dn);
-  out->n = n;
+  for (void* p : scratch) owl_dev_free(p);
+  if (e != cudaSuccess)
+    for (int i = 0; i < ntab; ++i) owl_sorted_free(&out[i]);
   return e;
 }
 
@@ -304,6 +426,149 @@ cudaError_t owl_diff_sorted(const SortedTable& a, const SortedTable& b, std::vec
   owl_dev_free(fa); owl_dev_free(fb); owl_dev_free(cboa); owl_dev_free(ia); owl_dev_free(ib);
   owl_dev_free(nsel); owl_dev_free(da); owl_dev_free(db); owl_dev_free(dt);
   return e;
+}
+
+namespace {
+
+__device__ __forceinline__ bool key_lt(const Key128& a, const Key128& b) {
+  return a.hi < b.hi || (a.hi == b.hi && a.lo < b.lo);
+}
+
+/* number of selected keys (k[idx[0..n)]) less than q */
+__device__ uint64_t count_less(const Key128* k, const uint64_t* idx, uint64_t n, const Key128& q) {
+  uint64_t lo = 0, hi = n;
+  while (lo < hi) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (key_lt(k[idx[mid]], q)) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+__global__ void diff_base_kernel(const unsigned long long* nsel, int ntab, unsigned long long* base) {
+  unsigned long long b = 0;
+  for (int t = 0; t < ntab; ++t) {
+    base[t] = b;
+    b += nsel[2 * t] + nsel[2 * t + 1];
+  }
+  base[ntab] = b;
+}
+
+/* the differing cells of table t as owl_diff rows, in canonical order: A-side rows (in B with another count,
+   or absent from B) and B-only rows merged by key (binary search of each in the other list) */
+__global__ void diff_rows_kernel(int t, const Key128* ak, const unsigned long long* ac, const unsigned long long* cboa,
+                                 const uint64_t* ia, const Key128* bk, const unsigned long long* bc, const uint64_t* ib,
+                                 const unsigned long long* nsel, const unsigned long long* base, owl_diff* out) {
+  const uint64_t nA = nsel[2 * t], nB = nsel[2 * t + 1];
+  const uint32_t NA = 0xFFFFFFFFu;
+  for (uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; r < nA + nB; r += (uint64_t)gridDim.x * blockDim.x) {
+    Key128 k;
+    unsigned long long ca, cb;
+    uint64_t pos;
+    if (r < nA) {
+      const uint64_t i = ia[r];
+      k = ak[i];
+      ca = ac[i];
+      cb = cboa[i];
+      pos = r + count_less(bk, ib, nB, k);
+    } else {
+      const uint64_t i = ib[r - nA];
+      k = bk[i];
+      ca = 0;
+      cb = bc[i];
+      pos = (r - nA) + count_less(ak, ia, nA, k);
+    }
+    owl_diff d;
+    d.table = (uint32_t)t;
+    d.bb = d.ins = d.j = d.prev = d.next = NA;
+    d._pad = 0;
+    d.x = 0;
+    if (t == T_ADDR) {
+      d.slot = (uint32_t)(k.hi >> 48);
+      d.bb = (uint32_t)((k.hi >> 30) & 0x3FFFFu);
+      d.ins = (uint32_t)((k.hi >> 22) & 0xFFu);
+      d.j = (uint32_t)(k.hi & OWL_MAX_J);
+      d.x = k.lo;
+    } else {
+      d.slot = (uint32_t)(k.hi >> 32);
+      const uint32_t a = (uint32_t)k.hi, b = (uint32_t)(k.lo >> 32), c = (uint32_t)k.lo;
+      if (t == T_NODE) d.bb = a;
+      else if (t == T_EDGE) { d.prev = a; d.next = c; }
+      else { d.bb = a; d.prev = b; d.next = c; }
+    }
+    d.count_a = ca;
+    d.count_b = cb;
+    out[base[t] + pos] = d;
+  }
+}
+
+}  // namespace
+
+/* A5 over all tables at once: the rows of every table in canonical (table, key) order, returned in host
+   memory allocated with malloc (caller frees); two host synchronisations in all. */
+cudaError_t owl_diff_rows(const SortedTable* A, const SortedTable* B, int ntab, owl_diff** rows, uint64_t* n_rows,
+                          size_t extra_rows, cudaStream_t st) {
+  *rows = nullptr;
+  *n_rows = 0;
+  std::vector<void*> scratch;
+  auto alloc = [&](size_t bytes) { void* p = owl_dev_alloc(bytes); scratch.push_back(p); return p; };
+  unsigned long long* nsel = (unsigned long long*)alloc(2 * ntab * 8 + 8);
+  unsigned long long* base = (unsigned long long*)alloc((ntab + 1) * 8);
+  cudaError_t e = (nsel && base) ? cudaSuccess : cudaErrorMemoryAllocation;
+  if (e == cudaSuccess) e = cudaMemsetAsync(nsel, 0, 2 * ntab * 8, st);
+  uint64_t max_rows = 0;
+  std::vector<unsigned char*> fa(ntab), fb(ntab);
+  std::vector<unsigned long long*> cboa(ntab);
+  std::vector<uint64_t*> ia(ntab), ib(ntab);
+  for (int t = 0; t < ntab && e == cudaSuccess; ++t) {
+    const uint64_t na = A[t].n, nb = B[t].n;
+    max_rows += na + nb;
+    fa[t] = (unsigned char*)alloc(na + 1);
+    fb[t] = (unsigned char*)alloc(nb + 1);
+    cboa[t] = (unsigned long long*)alloc((na + 1) * 8);
+    ia[t] = (uint64_t*)alloc((na + 1) * 8);
+    ib[t] = (uint64_t*)alloc((nb + 1) * 8);
+    if (!fa[t] || !fb[t] || !cboa[t] || !ia[t] || !ib[t]) { e = cudaErrorMemoryAllocation; break; }
+    if (na || nb)
+      diff_flag_kernel<<<grid_for(na > nb ? na : nb, 256), 256, 0, st>>>(A[t].k, A[t].c, na, B[t].k, B[t].c, nb, fa[t],
+                                                                           cboa[t], fb[t]);
+    size_t tmp = 0, tmp2 = 0;
+    cub::DeviceSelect::Flagged(nullptr, tmp, thrust::counting_iterator<uint64_t>(0), fa[t], ia[t], nsel + 2 * t, (int64_t)na, st);
+    cub::DeviceSelect::Flagged(nullptr, tmp2, thrust::counting_iterator<uint64_t>(0), fb[t], ib[t], nsel + 2 * t + 1, (int64_t)nb, st);
+    void* dt = alloc(tmp > tmp2 ? tmp : tmp2);
+    if (!dt) { e = cudaErrorMemoryAllocation; break; }
+    if (na) e = cub::DeviceSelect::Flagged(dt, tmp, thrust::counting_iterator<uint64_t>(0), fa[t], ia[t], nsel + 2 * t, (int64_t)na, st);
+    if (e == cudaSuccess && nb)
+      e = cub::DeviceSelect::Flagged(dt, tmp2, thrust::counting_iterator<uint64_t>(0), fb[t], ib[t], nsel + 2 * t + 1, (int64_t)nb, st);
+  }
+  owl_diff* drows = nullptr;
+  if (e == cudaSuccess) {
+    drows = (owl_diff*)alloc((max_rows + 1) * sizeof(owl_diff));
+    if (!drows) e = cudaErrorMemoryAllocation;
+  }
+  if (e == cudaSuccess) {
+    diff_base_kernel<<<1, 1, 0, st>>>(nsel, ntab, base);
+    for (int t = 0; t < ntab; ++t)
+      if (A[t].n + B[t].n)
+        diff_rows_kernel<<<grid_for(A[t].n + B[t].n, 256), 256, 0, st>>>(t, A[t].k, A[t].c, cboa[t], ia[t], B[t].k, B[t].c,
+                                                                          ib[t], nsel, base, drows);
+  }
+  unsigned long long total = 0;
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&total, base + ntab, 8, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e == cudaSuccess) {
+    *rows = (owl_diff*)malloc((total + extra_rows + 1) * sizeof(owl_diff));
+    if (!*rows) e = cudaErrorMemoryAllocation;
+  }
+  if (e == cudaSuccess && total) e = cudaMemcpyAsync(*rows, drows, total * sizeof(owl_diff), cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  for (void* p : scratch) owl_dev_free(p);
+  if (e != cudaSuccess) {
+    free(*rows);
+    *rows = nullptr;
+    return e;
+  }
+  *n_rows = total;
+  return cudaSuccess;
 }
 
 cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, uint4* out, uint64_t* perm,
