@@ -38,6 +38,17 @@ def _peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def _traffic(records_per_launch):
+    """DRAM bytes (read + write) per fold launch from the committed ncu --set full capture
+    (profiles/fold_traffic.json, written from the capture named there), scaled to this launch's records."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "fold_traffic.json")) as f:
+            t = json.load(f)
+        return t["traffic_bytes_per_launch"] / t["records_per_launch"] * records_per_launch
+    except Exception:  # noqa: BLE001
+        return None
+
+
 class ClockSampler:
     """nvidia-smi clocks / throttle reasons sampled during the timed region."""
 
@@ -331,7 +342,7 @@ def run_ours(args):
                    "parallelism": f"dp{world} (runs sharded, key-hash exchange)" if world > 1 else "single GPU",
                    "generate_s_untimed": round(t_gen, 2)},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": None, "kernel": "fold_kernel",
+                     "traffic": _traffic(fold_bytes / 16.0), "kernel": "fold_kernel",
                      "note": f"16 B/record algorithmic; {st['fold_launches']} fold launches, "
                              f"{fold_ms:.2f} ms avg (CUDA events on the launch stream); peak {peak_src}"},
         "clocks": ck,

@@ -397,7 +397,7 @@ owl_status build_tables(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTa
       return s;
     }
     if (!overflow) {
-      /* next builds: at most 1/16 of the address cells claimed, so nearly every key sits in its home
+      /* next builds: at most 1/8 of the address cells claimed (load shift 3, profiles/r01_v4_ab.txt), so nearly every key sits in its home
          bucket and the fold's first probe hits (owl_fold.cu) */
       unsigned long long fill = 0;
       cudaMemcpy(&fill, tab[T_ADDR].fill, sizeof fill, cudaMemcpyDeviceToHost);
