@@ -50,9 +50,7 @@ using namespace owl_dev;
 #define FOLD_THREADS (FOLD_WARPS * 32)
 #define CFK 128      /* shared cells per CF table kind (node, edge, triple) */
 #define CFK_LIMIT 96
-#ifndef VCAP
-#define VCAP 64     /* per-warp overflow visit map (BBs beyond the 32 held in registers) */
-#endif
+#define VCAP 1024    /* per-warp overflow visit map in global scratch (BBs beyond the 32 held in registers) */
 #define VGEN_MAX 0x3FFFu /* visit-map entry = gen<<18 | bb: a new generation per traced warp, 0 = empty */
 #ifndef PF_LOG
 #define PF_LOG 12    /* L2 bulk prefetch granule: 4 KB (256 records) */
@@ -93,6 +91,10 @@ namespace {
 /* per-warp fields read only at traced-warp / tile boundaries, in the slow path and on errors */
 struct RunDesc {
   const uint4* rec; /* segment base */
+  uint32_t* vk;     /* overflow visit map of this warp (global scratch): VCAP keys, then VCAP counts */
+  const uint4* tile_end; /* traced warps starting at or after this belong to the next tile */
+  uint32_t prev, curj;   /* walk context read only at BB entries (cur and khi stay in registers) */
+  uint32_t gen;          /* generation of the traced warp in the overflow visit map */
   uint32_t* seen;
   uint32_t slot, n_warps, seg_index;
 };
@@ -102,8 +104,6 @@ struct __align__(16) FoldSmem {
   ulonglong2 dir_key[DIRCAP]; /* (attribute key hi, x) broadcast cell, or (hi, x>>10 | PAGE_TAG) window */
   uint32_t dir_val[DIRCAP];
   uint32_t filt[1 << FILTER_LOG]; /* 4-way buckets of tag<<8 | sightings of keys not in the directory */
-  uint32_t vkey[FOLD_WARPS][VCAP]; /* per-warp visit maps: gen<<18 | bb, and the visit count */
-  uint32_t vcnt[FOLD_WARPS][VCAP];
   uint16_t page_dir[NPAGE];   /* page -> directory slot (final flush) */
   ulonglong2 cf_key[3][CFK];  /* node / edge / triple cells, one table per kind */
   unsigned int cf_cnt[3][CFK];
@@ -335,16 +335,15 @@ enum { W_INWARP = 2u, W_SKIP = 4u };
 struct Walker {
   const uint4* p;  /* next record */
   uint64_t khi;    /* slot<<48 | cur<<30 | curj: address key of the current context (ins added per chunk) */
-  uint32_t g0, cur, prev, curj, slot;
+  uint32_t g0, cur;
   uint32_t want;   /* meta of a fast-path record modulo lane and ins: MEM | cur<<8 (impossible when skipping) */
   uint32_t st;
-  uint32_t gen;    /* generation of the traced warp in the shared overflow visit map */
   uint32_t vb, vn; /* visit map in registers: lane l holds BB vb and its visit count vn (32 BBs / warp) */
 };
 
 /* visits[b] += 1 for the traced warp; returns the new visit ordinal j (reading R8).  The first
    32 distinct BBs of a traced warp live in registers (one per lane), further ones in the shared map. */
-__device__ __forceinline__ uint32_t visit(Walker& w, uint32_t* vk, uint32_t* vc, uint32_t b, int lane,
+__device__ __forceinline__ uint32_t visit(Walker& w, const RunDesc& d, uint32_t b, int lane,
                                           FoldStatus* st) {
   const unsigned m = __ballot_sync(FULL, w.vb == b);
   if (m) {
@@ -361,7 +360,8 @@ __device__ __forceinline__ uint32_t visit(Walker& w, uint32_t* vk, uint32_t* vc,
     }
     return 1;
   }
-  return visits_inc(vk, vc, b, w.gen, lane, st);
+  uint32_t* vk = d.vk;
+  return visits_inc(vk, vk + VCAP, b, d.gen, lane, st);
 }
 
 struct SlowRes {
@@ -374,7 +374,7 @@ struct SlowRes {
 /* noinline (and everything by value): the slow path is rare, and keeping it out of the unrolled fast
    loop keeps the kernel within the instruction cache */
 __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Walker w, RunDesc& d,
-                                           const FoldArgs& a, FoldSmem& s, uint32_t* vk, uint32_t* vc,
+                                           const FoldArgs& a, FoldSmem& s,
                                            const int lane) {
   bool good;
   uint64_t khi_out, lo_out;
@@ -393,11 +393,11 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
     const bool bbbad = isbb && (addr != 0 || (meta & 0x7C0000FFu) != 0);
     if (bbbad) report(a.status, d.seg_index, idx, KERR_BBFIELDS);
     const unsigned bbmask = __ballot_sync(FULL, isbb && !bbbad);
-    const uint32_t cur0 = w.cur, j0 = w.curj;
+    const uint32_t cur0 = w.cur, j0 = d.curj;
     uint32_t myj = 0;
     if (bbmask) {
-      uint32_t prev = w.prev, curj = j0;
-      const uint64_t slot_hi = (uint64_t)w.slot << 32;
+      uint32_t prev = d.prev, curj = j0;
+      const uint64_t slot_hi = (uint64_t)d.slot << 32;
       unsigned m = bbmask;
       while (m) {
         const int k = __ffs(m) - 1;
@@ -412,14 +412,15 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
         }
         if (w.cur != OWL_NONE_BB) prev = w.cur;
         w.cur = b;
-        curj = visit(w, vk, vc, b, lane, a.status);
+        curj = visit(w, d, b, lane, a.status);
         if (lane == k) myj = curj;
       }
-      w.khi = ((uint64_t)w.slot << 48) | ((uint64_t)w.cur << 30) | (uint64_t)curj;
+      w.khi = ((uint64_t)d.slot << 48) | ((uint64_t)w.cur << 30) | (uint64_t)curj;
       w.want = 0x80000000u | (w.cur << 8);
       if (curj > OWL_MAX_J && lane == 0) atomicOr(&a.status->limit, 1u);
-      w.prev = prev;
-      w.curj = curj;
+      __syncwarp();
+      d.prev = prev; /* every lane writes the same value */
+      d.curj = curj;
       nproc = 32 - __clz(bbmask); /* consume up to the last BB_ENTRY: the next chunk starts aligned */
     }
     const bool ismem = lane < nproc && (meta >> 31) != 0;
@@ -440,15 +441,15 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
     }
     good = ismem && code == 0;
     if (good && cj > OWL_MAX_J) atomicOr(&a.status->limit, 1u);
-    khi_out = ((uint64_t)w.slot << 48) | ((uint64_t)cbb << 30) | ((uint64_t)ins << 22) | cj;
+    khi_out = ((uint64_t)d.slot << 48) | ((uint64_t)cbb << 30) | ((uint64_t)ins << 22) | cj;
     lo_out = addr;
   }
   w.p += nproc;
   if (nvalid < 32 && nproc == nvalid) { /* warp end: last BB -> S */
     if (a.mode == 0 && !(w.st & W_SKIP) && w.cur != OWL_NONE_BB && (lane == T_EDGE || lane == T_TRIPLE)) {
-      const uint64_t hi = ((uint64_t)w.slot << 32) | w.cur;
+      const uint64_t hi = ((uint64_t)d.slot << 32) | w.cur;
       if (lane == T_EDGE) cf_insert(s, a, T_EDGE, hi, OWL_SENTINEL);
-      else cf_insert(s, a, T_TRIPLE, hi, ((uint64_t)w.prev << 32) | OWL_SENTINEL);
+      else cf_insert(s, a, T_TRIPLE, hi, ((uint64_t)d.prev << 32) | OWL_SENTINEL);
     }
     w.st &= ~W_INWARP;
   }
@@ -461,7 +462,7 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
   return res;
 }
 
-__device__ __forceinline__ void begin_traced_warp(Walker& w, RunDesc& d, const FoldArgs& a, uint32_t* vk,
+__device__ __forceinline__ void begin_traced_warp(Walker& w, RunDesc& d, const FoldArgs& a,
                                                   int lane) {
   w.g0 = __ldg(&w.p->z);
   w.st = W_INWARP;
@@ -473,13 +474,17 @@ __device__ __forceinline__ void begin_traced_warp(Walker& w, RunDesc& d, const F
     if (atomicOr(&d.seen[w.g0 >> 5], bit) & bit)
       atomicMin(&a.status->not_warp_major, ((unsigned long long)d.seg_index << 32) | w.g0);
   }
-  if (++w.gen > VGEN_MAX) { /* generations wrapped: clear the map */
-    for (int i = lane; i < VCAP; i += 32) vk[i] = 0;
-    w.gen = 1;
+  __syncwarp();
+  uint32_t gen = d.gen + 1;
+  if (gen > VGEN_MAX) { /* generations wrapped: clear the map */
+    for (int i = lane; i < VCAP; i += 32) d.vk[i] = 0;
+    gen = 1;
   }
   __syncwarp();
-  w.prev = OWL_SENTINEL;
-  w.curj = 0;
+  d.gen = gen; /* every lane writes the same values */
+  d.prev = OWL_SENTINEL;
+  d.curj = 0;
+  __syncwarp();
   w.vb = 0xFFFFFFFFu;
   w.vn = 0;
   w.cur = OWL_NONE_BB;
@@ -534,9 +539,15 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     s.dir_key[i] = make_ulonglong2(OWL_EMPTY_KEY, OWL_EMPTY_KEY);
     s.dir_val[i] = 0;
   }
-  uint32_t* vk = s.vkey[warp];
-  uint32_t* vc = s.vcnt[warp];
-  for (int i = lane; i < VCAP; i += 32) vk[i] = 0;
+  /* overflow visit map of this warp (global scratch, L1-cached; only this warp touches it) */
+  {
+    uint32_t* vk = args.vmap + ((size_t)blockIdx.x * FOLD_WARPS + warp) * (2 * VCAP);
+    for (int i = lane; i < VCAP; i += 32) vk[i] = 0;
+    if (lane == 0) {
+      s.rd[warp].vk = vk;
+      s.rd[warp].gen = 0;
+    }
+  }
   for (int i = threadIdx.x; i < (1 << FILTER_LOG); i += FOLD_THREADS) s.filt[i] = 0;
   __syncthreads();
   const uint64_t pol = evict_first_policy();
@@ -545,7 +556,6 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
   const uint32_t shift = tab_shift(tab.cap);
   RunDesc& d = s.rd[warp];
   uint32_t claims = 0;
-  uint32_t gen = 0;
 #ifdef OWL_FOLD_STATS
   unsigned long long stat[8] = {0, 0, 0, 0, 0, 0, 0, 0};
 #endif
@@ -571,7 +581,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
       d.seg_index = sg.seg_index;
     }
     const uint4* const end = sg.rec + sg.n;
-    const uint4* const tile_end = sg.rec + e;
+    if (lane == 0) d.tile_end = sg.rec + e;
     Walker w;
     w.p = sg.rec + first_warp_start(sg.rec, b, e, lane);
     const uint4* p_acc = w.p; /* records walked since the last accounting */
@@ -579,10 +589,6 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     w.g0 = w.cur = 0;
     w.khi = 0;
     w.want = 1u;
-    w.gen = gen;
-    w.slot = sg.slot;
-    w.prev = OWL_SENTINEL;
-    w.curj = 0;
     w.vb = 0xFFFFFFFFu;
     w.vn = 0;
     /* shared counting stays open while the CTA's walked records cannot wrap a 32-bit counter */
@@ -598,8 +604,8 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
 
     for (;;) {
       if (!(w.st & W_INWARP)) {
-        if (w.p >= tile_end) break;
-        begin_traced_warp(w, d, a, vk, lane);
+        if (w.p >= d.tile_end) break;
+        begin_traced_warp(w, d, a, lane);
       }
       if ((uint64_t)(w.p - p_acc) > (1ull << 22)) { /* very long traced warp: account as we go */
         if (lane == 0) {
@@ -722,25 +728,27 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
              boundaries).  Consume it alone, then realign the rest of the step. */
           STAT(1);
           const uint32_t b = (__shfl_sync(FULL, r.w, 0) >> 8) & 0x3FFFFu;
-          const uint64_t slot_hi = (uint64_t)w.slot << 32;
+          const uint64_t slot_hi = (uint64_t)d.slot << 32;
           if (lane < 3) { /* node / edge / triple cell of this entry, one lane (and table) each */
             const bool first = w.cur == OWL_NONE_BB;
             const uint64_t hi = slot_hi | (lane == T_NODE ? b : (first ? OWL_SENTINEL : w.cur));
-            const uint64_t lo = lane == T_NODE ? 0 : (lane == T_EDGE ? (uint64_t)b : (((uint64_t)w.prev << 32) | b));
+            const uint64_t lo = lane == T_NODE ? 0 : (lane == T_EDGE ? (uint64_t)b : (((uint64_t)d.prev << 32) | b));
             if (lane != T_TRIPLE || !first) cf_insert(s, a, lane, hi, lo);
           }
-          if (w.cur != OWL_NONE_BB) w.prev = w.cur;
+          __syncwarp();
+          if (w.cur != OWL_NONE_BB) d.prev = w.cur; /* every lane writes the same value */
           w.cur = b;
-          w.curj = visit(w, vk, vc, b, lane, a.status);
-          if (w.curj > OWL_MAX_J && lane == 0) atomicOr(&a.status->limit, 1u);
-          w.khi = ((uint64_t)w.slot << 48) | ((uint64_t)b << 30) | (uint64_t)w.curj;
+          const uint32_t j = visit(w, d, b, lane, a.status);
+          d.curj = j;
+          if (j > OWL_MAX_J && lane == 0) atomicOr(&a.status->limit, 1u);
+          w.khi = ((uint64_t)d.slot << 48) | ((uint64_t)b << 30) | (uint64_t)j;
           w.want = 0x80000000u | (b << 8);
           w.p += 1;
 #pragma unroll
           for (int c = FOLD_U - 1; c > u; --c) rr[c] = funnel(rr[c - 1], rr[c], 1, lane);
         } else {
           STAT(1);
-          const SlowRes sr = slow_chunk(r, __ballot_sync(FULL, r.z == w.g0 && w.p + lane < end), w, d, a, s, vk, vc,
+          const SlowRes sr = slow_chunk(r, __ballot_sync(FULL, r.z == w.g0 && w.p + lane < end), w, d, a, s,
                                         lane);
           w = sr.w;
           lead[u] = sr.good;
@@ -783,7 +791,6 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
           if (lead[u]) claims += addr_insert_slow(tab, home[u], khi[u], klo[u], cnt[u], a.status);
       }
     }
-    gen = w.gen;
     /* records walked by this item bound every shared counter it touched */
     if (lane == 0) {
       const unsigned long long n = (unsigned long long)(w.p - p_acc);
@@ -833,6 +840,8 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
 
 int owl_fold_ctas_per_sm() { return 1; }
 int owl_fold_runs_per_warp() { return 1; }
+size_t owl_fold_scratch_bytes(int grid) { return (size_t)grid * FOLD_WARPS * 2 * VCAP * sizeof(uint32_t); }
+int owl_fold_max_bbs() { return 32 + VCAP; }
 
 cudaError_t owl_launch_fold(const FoldArgs& a, int grid, cudaStream_t st) {
   const size_t smem = sizeof(FoldSmem);

@@ -319,8 +319,10 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     a.mode = getenv("OWL_FOLD_MODE") ? (uint32_t)atoi(getenv("OWL_FOLD_MODE")) : 0u;
     const int per_sm = ctx->cfg.fold_ctas_per_sm ? (int)ctx->cfg.fold_ctas_per_sm : owl_fold_ctas_per_sm();
     const int grid = ctx->n_sm * per_sm;
+    a.vmap = (uint32_t*)owl_dev_alloc(owl_fold_scratch_bytes(grid));
+    scratch.push_back(a.vmap);
     cudaEventRecord(ctx->ev0, st);
-    cudaError_t e = items ? owl_launch_fold(a, grid, st) : cudaSuccess;
+    cudaError_t e = !a.vmap ? cudaErrorMemoryAllocation : items ? owl_launch_fold(a, grid, st) : cudaSuccess;
     cudaEventRecord(ctx->ev1, st);
     if (e == cudaSuccess) e = cudaMemcpyAsync(&hs, ctx->d_status, sizeof hs, cudaMemcpyDeviceToHost, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
@@ -361,8 +363,9 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
                     "segment (run %u, seq %u) is flagged OWL_SEG_WARP_MAJOR but warp %u's records are not contiguous",
                     plan[si].s.run, plan[si].s.seq, (uint32_t)hs.not_warp_major);
     } else if (hs.limit) {
-      status = fail(OWL_ERR_CAPACITY, (hs.limit & 2) ? "a traced warp visits more than 256 distinct basic blocks"
-                                                     : "a basic-block visit ordinal j exceeds 2^22-1");
+      status = (hs.limit & 2) ? fail(OWL_ERR_CAPACITY, "a traced warp visits more than %d distinct basic blocks",
+                                     owl_fold_max_bbs())
+                              : fail(OWL_ERR_CAPACITY, "a basic-block visit ordinal j exceeds 2^22-1");
     }
     *overflow = hs.overflow;
   }

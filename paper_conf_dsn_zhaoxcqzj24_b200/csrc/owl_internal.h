@@ -95,6 +95,7 @@ struct FoldArgs {
   uint64_t n_items;
   DevTable tab[T_NUM];
   FoldStatus* status;
+  uint32_t* vmap; /* per-warp overflow visit maps (owl_fold_scratch_bytes(grid) bytes of device scratch) */
   uint32_t mode; /* experiment switch (OWL_FOLD_MODE): 0 normal, 1 no address inserts, 2 stream only */
 };
 
@@ -102,6 +103,8 @@ struct FoldArgs {
 cudaError_t owl_launch_fold(const FoldArgs& a, int grid, cudaStream_t st);
 int owl_fold_ctas_per_sm();
 int owl_fold_runs_per_warp();
+size_t owl_fold_scratch_bytes(int grid);
+int owl_fold_max_bbs(); /* distinct BBs one traced warp may visit */
 
 struct Key128 {
   unsigned long long hi, lo;

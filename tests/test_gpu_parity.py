@@ -268,3 +268,71 @@ def test_work_queue_stress_long_warps(ctx):
             assert np.array_equal(ev[t]["count"], 40 * o[t]["count"]), t
     finally:
         ctx.forget_runs(runs)
+
+
+def _build_one(ctx, rec, n_warps, flags=None):
+    buf = torch.from_numpy(rec.view(np.uint8).copy()).cuda()
+    seg = api.Segment(0, 0, 0, n_warps, 10, buf, len(rec)) if flags is None else \
+        api.Segment(0, 0, 0, n_warps, 10, buf, len(rec), flags=flags)
+    ctx.ingest([seg])
+    try:
+        return ctx.build([0]).export()
+    finally:
+        ctx.forget_runs([0])
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_traces_parity(ctx, seed):
+    """Random valid traces (random active-lane subsets, so chunks straddle instructions; small address pools,
+    so broadcast / window / scattered chunks mix; repeated BBs): GPU = oracle, warp-major and interleaved."""
+    rng = np.random.default_rng(1000 + seed)
+    n_warps = int(rng.integers(1, 40))
+    rec = H.random_trace(rng, n_warps=n_warps, max_bbs=int(rng.integers(1, 30)), n_bb_ids=int(rng.integers(1, 12)),
+                         max_ins=int(rng.integers(1, 6)), n_addr=int(rng.integers(1, 600)),
+                         active=float(rng.uniform(0.3, 1.0)))
+    if len(rec) == 0:
+        return
+    want = oracle.build([oracle.Segment(0, 0, 0, n_warps, 10, rec)]).export()
+    assert _build_one(ctx, rec, n_warps) == want
+    assert _build_one(ctx, H.interleave_random(rng, rec), n_warps, flags=0) == want
+
+
+def test_many_distinct_bbs(ctx):
+    """Traced warps visiting up to 700 distinct BBs (beyond the 32 held in registers: the overflow visit map),
+    several times each, so j counts per BB; one more distinct BB than the fold supports is a capacity error."""
+    rng = np.random.default_rng(7)
+    rows = []
+    for w in range(6):
+        bbs = rng.permutation(5000)[: 100 * (w + 1) + 1]
+        for rep in range(3):
+            for b in bbs:
+                rows.append(H.bb_rec(w, int(b)))
+                for lane in range(0, 32, 3):
+                    rows.append(H.mem_rec(w, int(b), rep, lane, (3 << 60) | int(rng.integers(0, 64)) * 4))
+    rec = H.to_records(rows)
+    want = oracle.build([oracle.Segment(0, 0, 0, 6, 10, rec)]).export()
+    assert _build_one(ctx, rec, 6) == want
+    limit = 32 + 1024  # register visit map + overflow map (owl_fold.cu VCAP; DESIGN.md §5 limits)
+    over = H.to_records([H.bb_rec(0, b) for b in range(limit + 1)])
+    with pytest.raises(api.OwlError, match="OWL_ERR_CAPACITY"):
+        _build_one(ctx, over, 1)
+
+
+def test_wide_keys_sort_fallback(ctx):
+    """More than 64 key bits vary across the address table (random 60-bit addresses, every ins and many j):
+    the canonical sort takes the full 128-bit path; tables and diff still match the oracle."""
+    rng = np.random.default_rng(11)
+    rows = []
+    for w in range(8):
+        for v in range(40):
+            b = int(rng.integers(0, 3))
+            rows.append(H.bb_rec(w, b))
+            for ins in range(int(rng.integers(1, 4))):
+                i = int(rng.integers(0, 256))
+                for lane in range(32):
+                    x = (int(rng.integers(0, 9)) << 60) | int(rng.integers(0, 1 << 60))
+                    rows.append(H.mem_rec(w, b, i, lane, x))
+    rec = H.to_records(rows)
+    of = oracle.build([oracle.Segment(0, 0, 0, 8, 10, rec)])
+    assert _build_one(ctx, rec, 8) == of.export()
+    assert H.parse_blob(of.export())["addr"].shape[0] > 4096
