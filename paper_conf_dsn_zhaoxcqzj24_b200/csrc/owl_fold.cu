@@ -95,6 +95,7 @@ struct RunDesc {
   const uint4* tile_end; /* traced warps starting at or after this belong to the next tile */
   uint32_t prev, curj;   /* walk context read only at BB entries (cur and khi stay in registers) */
   uint32_t gen;          /* generation of the traced warp in the overflow visit map */
+  const uint4* p_acc;    /* records walked since the last accounting start here */
   uint32_t* seen;
   uint32_t slot, n_warps, seg_index;
 };
@@ -550,10 +551,9 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
   }
   for (int i = threadIdx.x; i < (1 << FILTER_LOG); i += FOLD_THREADS) s.filt[i] = 0;
   __syncthreads();
-  const uint64_t pol = evict_first_policy();
   const uint64_t tile = 1ull << a.tile_shift;
-  const DevTable tab = a.tab[T_ADDR];
-  const uint32_t shift = tab_shift(tab.cap);
+  owl_bucket* const tab_b = a.tab[T_ADDR].b; /* the rest of the table descriptor is read from shared */
+  const uint32_t shift = tab_shift(a.tab[T_ADDR].cap);
   RunDesc& d = s.rd[warp];
   uint32_t claims = 0;
 #ifdef OWL_FOLD_STATS
@@ -584,7 +584,8 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     if (lane == 0) d.tile_end = sg.rec + e;
     Walker w;
     w.p = sg.rec + first_warp_start(sg.rec, b, e, lane);
-    const uint4* p_acc = w.p; /* records walked since the last accounting */
+    uint32_t steps = 0; /* steps since the last accounting (a step walks <= 32 * FOLD_U records) */
+    if (lane == 0) d.p_acc = w.p;
     w.st = 0;
     w.g0 = w.cur = 0;
     w.khi = 0;
@@ -607,16 +608,19 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         if (w.p >= d.tile_end) break;
         begin_traced_warp(w, d, a, lane);
       }
-      if ((uint64_t)(w.p - p_acc) > (1ull << 22)) { /* very long traced warp: account as we go */
+      if (++steps >= (1u << 16)) { /* very long traced warp: account as we go */
+        __syncwarp();
         if (lane == 0) {
-          const unsigned long long n = (unsigned long long)(w.p - p_acc);
+          const unsigned long long n = (unsigned long long)(w.p - d.p_acc);
           if (atomicAdd(&s.walked, n) + n > SHARED_TOTAL_LIMIT) s.off = 1;
+          d.p_acc = w.p;
         }
         __syncwarp();
-        p_acc = w.p;
+        steps = 0;
         shared_on = !*(volatile unsigned int*)&s.off;
       }
       uint4 rr[FOLD_U];
+      const uint64_t pol = evict_first_policy(); /* one instruction: cheaper than a live register pair */
       if (w.p + 32 * FOLD_U <= end) {
 #pragma unroll
         for (int u = 0; u < FOLD_U; ++u) rr[u] = ld_stream(w.p + u * 32 + lane, pol);
@@ -773,7 +777,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
 #pragma unroll
       for (int u = 0; u < FOLD_U; ++u) {
         home[u] = tab_index(khi[u], klo[u], shift);
-        kk[u] = ld_bucket_keys_if(lead[u], tab.b + (home[u] >> 1));
+        kk[u] = ld_bucket_keys_if(lead[u], tab_b + (home[u] >> 1));
       }
       unsigned miss_any = 0;
 #pragma unroll
@@ -781,19 +785,20 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         const bool h0 = kk[u].x == khi[u] && kk[u].y == klo[u];
         const bool h1 = kk[u].z == khi[u] && kk[u].w == klo[u];
         const bool hit = lead[u] && (h0 || h1);
-        red_add_if(hit, &tab.b[home[u] >> 1].count[h1 ? 1 : 0], cnt[u]);
+        red_add_if(hit, &tab_b[home[u] >> 1].count[h1 ? 1 : 0], cnt[u]);
         lead[u] = lead[u] && !hit; /* now: missed (absent, or displaced past the home bucket) */
         miss_any |= __ballot_sync(FULL, lead[u]);
       }
       if (miss_any) {
 #pragma unroll
         for (int u = 0; u < FOLD_U; ++u)
-          if (lead[u]) claims += addr_insert_slow(tab, home[u], khi[u], klo[u], cnt[u], a.status);
+          if (lead[u]) claims += addr_insert_slow(a.tab[T_ADDR], home[u], khi[u], klo[u], cnt[u], a.status);
       }
     }
     /* records walked by this item bound every shared counter it touched */
+    __syncwarp();
     if (lane == 0) {
-      const unsigned long long n = (unsigned long long)(w.p - p_acc);
+      const unsigned long long n = (unsigned long long)(w.p - d.p_acc);
       if (atomicAdd(&s.walked, n) + n > SHARED_TOTAL_LIMIT) s.off = 1;
     }
     /* cells claimed by this item -> table fill; past the load limit the build stops and regrows */
@@ -801,6 +806,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
 #pragma unroll
       for (int o = 16; o; o >>= 1) claims += __shfl_xor_sync(FULL, claims, o);
       if (lane == 0) {
+        const DevTable& tab = a.tab[T_ADDR];
         const unsigned long long f = atomicAdd(tab.fill, (unsigned long long)claims) + claims;
         if (f > (tab.cap >> 1) + (tab.cap >> 2)) atomicOr(&a.status->overflow, 1u << T_ADDR);
         atomicAdd(&a.status->n_claim, (unsigned long long)claims);
@@ -821,13 +827,13 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     const uint32_t c = s.page[pg][b];
     if (c) {
       const ulonglong2 k = s.dir_key[s.page_dir[pg]];
-      g_insert(tab, T_ADDR, k.x, ((k.y & ~PAGE_TAG) << 10) | ((uint64_t)b << 2), c, a.status);
+      g_insert(a.tab[T_ADDR], T_ADDR, k.x, ((k.y & ~PAGE_TAG) << 10) | ((uint64_t)b << 2), c, a.status);
     }
   }
   for (int i = threadIdx.x; i < DIRCAP; i += FOLD_THREADS) {
     const ulonglong2 k = s.dir_key[i];
     const uint32_t c = s.dir_val[i];
-    if (k.x != OWL_EMPTY_KEY && (k.y & PAGE_TAG) != PAGE_TAG && c) g_insert(tab, T_ADDR, k.x, k.y, c, a.status);
+    if (k.x != OWL_EMPTY_KEY && (k.y & PAGE_TAG) != PAGE_TAG && c) g_insert(a.tab[T_ADDR], T_ADDR, k.x, k.y, c, a.status);
   }
   for (int i = threadIdx.x; i < 3 * CFK; i += FOLD_THREADS) {
     const int tbl = i / CFK;
