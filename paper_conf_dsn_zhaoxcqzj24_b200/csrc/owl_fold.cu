@@ -47,6 +47,13 @@ using namespace owl_dev;
 #ifndef FOLD_U
 #define FOLD_U 2 /* chunks of 32 records per warp and step */
 #endif
+/* experiment modes (OWL_FOLD_MODE at run time in -DFOLD_RUNTIME_MODE builds, tools/): 1 no global-table
+   inserts, 2 stream + walk only, 3 no L2 prefetch, 8 no shared counting; the product is mode 0 */
+#ifdef FOLD_RUNTIME_MODE
+#define FOLD_MODE_OF(a) ((a).mode)
+#else
+#define FOLD_MODE_OF(a) 0u
+#endif
 #define FOLD_THREADS (FOLD_WARPS * 32)
 #define CFK 128      /* shared cells per CF table kind (node, edge, triple) */
 #define CFK_LIMIT 96
@@ -404,7 +411,7 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
         const int k = __ffs(m) - 1;
         m &= m - 1;
         const uint32_t b = __shfl_sync(FULL, bbf, k);
-        if (a.mode == 0 && lane < 3) { /* node, edge, triple cell of this entry: one lane (and table) each */
+        if (FOLD_MODE_OF(a) == 0 && lane < 3) { /* node, edge, triple cell of this entry: one lane (and table) each */
           if (lane == T_NODE) cf_insert(s, a, T_NODE, slot_hi | b, 0);
           else if (lane == T_EDGE) /* S -> first BB, else cur -> b */
             cf_insert(s, a, T_EDGE, slot_hi | (w.cur == OWL_NONE_BB ? OWL_SENTINEL : w.cur), b);
@@ -447,7 +454,7 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
   }
   w.p += nproc;
   if (nvalid < 32 && nproc == nvalid) { /* warp end: last BB -> S */
-    if (a.mode == 0 && !(w.st & W_SKIP) && w.cur != OWL_NONE_BB && (lane == T_EDGE || lane == T_TRIPLE)) {
+    if (FOLD_MODE_OF(a) == 0 && !(w.st & W_SKIP) && w.cur != OWL_NONE_BB && (lane == T_EDGE || lane == T_TRIPLE)) {
       const uint64_t hi = ((uint64_t)d.slot << 32) | w.cur;
       if (lane == T_EDGE) cf_insert(s, a, T_EDGE, hi, OWL_SENTINEL);
       else cf_insert(s, a, T_TRIPLE, hi, ((uint64_t)d.prev << 32) | OWL_SENTINEL);
@@ -526,7 +533,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
   if (threadIdx.x == 0) {
     a = args;
     s.npages = 0;
-    s.off = args.mode == 8 ? 1u : 0u; /* experiment mode 8: global table only */
+    s.off = FOLD_MODE_OF(args) == 8 ? 1u : 0u; /* experiment mode 8: global table only */
     s.walked = 0;
   }
   if (threadIdx.x < 3) s.cf_fill[threadIdx.x] = 0;
@@ -594,7 +601,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     w.vn = 0;
     /* shared counting stays open while the CTA's walked records cannot wrap a 32-bit counter */
     bool shared_on = !*(volatile unsigned int*)&s.off;
-    if (lane < PF_DIST && a.mode != 3) { /* prime the L2 prefetch window */
+    if (lane < PF_DIST && FOLD_MODE_OF(a) != 3) { /* prime the L2 prefetch window */
       const char* q = (const char*)(((((uintptr_t)w.p) >> PF_LOG) + lane) << PF_LOG);
       if (q < (const char*)end) {
         const uint64_t left = (uint64_t)((const char*)end - q);
@@ -631,7 +638,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
           rr[u] = q < end ? ld_stream(q, pol) : make_uint4(0, 0, 0xFFFFFFFFu, 0);
         }
       }
-      if (a.mode != 3) { /* keep PF_DIST granules of the stream in flight to L2 */
+      if (FOLD_MODE_OF(a) != 3) { /* keep PF_DIST granules of the stream in flight to L2 */
         const uintptr_t g1 = ((uintptr_t)(w.p + 32 * FOLD_U)) >> PF_LOG;
         if (g1 != (((uintptr_t)w.p) >> PF_LOG) && lane == 0) {
           const char* q = (const char*)((g1 + PF_DIST - 1) << PF_LOG);
@@ -660,7 +667,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
           khi[u] = w.khi | ((uint64_t)(r.w & 0xFFu) << 22);
           klo[u] = ((uint64_t)r.y << 32) | r.x;
           lead[u] = true;
-          if (a.mode == 2) { /* experiment: stream + walk only */
+          if (FOLD_MODE_OF(a) == 2) { /* experiment: stream + walk only */
             lead[u] = false;
             continue;
           }
@@ -727,7 +734,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
             if (__any_sync(FULL, ready)) admit_ready(s, ready, khi[u], lo, h0, fi, !bc, lane);
           }
         } else if (__shfl_sync(FULL, r.z == w.g0 && (r.w & 0xFC0000FFu) == 0 && r.x == 0 && r.y == 0, 0) &&
-                   !(w.st & W_SKIP) && a.mode == 0) {
+                   !(w.st & W_SKIP) && FOLD_MODE_OF(a) == 0) {
           /* the common slow chunk: a well-formed BB_ENTRY in lane 0 (chunks start on instruction
              boundaries).  Consume it alone, then realign the rest of the step. */
           STAT(1);
@@ -770,7 +777,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         any_lead |= __ballot_sync(FULL, lead[u]);
 
       }
-      if (!any_lead || a.mode == 1) continue;
+      if (!any_lead || FOLD_MODE_OF(a) == 1) continue;
       /* global table: first probes of all chunks in flight together, predicated REDs, rare misses */
       uint32_t home[FOLD_U];
       ulonglong4 kk[FOLD_U];
