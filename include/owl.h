@@ -187,6 +187,21 @@ owl_status owl_adcfg_destroy(owl_adcfg* g);
  * (table, key).  Zero rows <=> identical traces (§VI). */
 owl_status owl_diff_adcfg(owl_ctx* ctx, const owl_adcfg* a, const owl_adcfg* b, owl_diff** rows, size_t* n_rows);
 
+/* ---- N1: input-class filtering -----------------------------------------------------
+ * "inputs that generate identical traces [are] the same class ... the program [is] side-channel
+ * leakage-free when there is only one class" (§VI).  Builds each run's A-DCFG (all of its
+ * ingested segments; their input_class is ignored) and partitions the runs by identical A-DCFGs (same
+ * kernel sequence, same node / edge / triple / address tables and counts).  Runs are visited in the
+ * given order; class ids are assigned in order of first appearance, so a class's representative is its
+ * first run (the paper picks one at random; reading R21).  class_of[i] receives the class of runs[i]
+ * (caller-allocated, n_runs entries); *n_classes the number of classes (1 <=> leakage-free for these
+ * inputs).  A 128-bit order-independent fingerprint of each run's cells buckets the runs on the device;
+ * every membership is then confirmed by an exact comparison with the representative (A5 with zero
+ * rows and equal slot tables), so the partition is exact.  Errors: INVALID_ARG (NULL, a run not
+ * ingested or repeated), MALFORMED_TRACE / CAPACITY as for the build, CUDA. */
+owl_status owl_filter_inputs(owl_ctx* ctx, const uint32_t* runs, size_t n_runs, uint32_t* class_of,
+                             uint32_t* n_classes);
+
 /* ---- A6-A7: leakage test ------------------------------------------------------------------------
  * Kernel test, then for every aligned slot pair one KS test (Eqs. 1-4) per node's
  * H_cf (Eqs. 5-8) and per (bb, ins, j) H_addr, both sides present.  A test fails

@@ -149,3 +149,17 @@ def run_config(params, runs=None, threads: int = 0):
             by_cls[m.input_class].append(Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, rec))
     t_gen = time.perf_counter() - t_gen
     return by_cls, t_gen
+
+
+def filter_inputs(segments_by_run, threads: int = 0):
+    """N1, input-class filtering (§VI): "inputs that generate identical traces [are] the same
+    class".  The plain definition: build each run's A-DCFG (its segments, one input class for all) and
+    group the runs whose canonical dumps are byte-identical, classes numbered in order of first
+    appearance.  segments_by_run: list of (run, [Segment]) in the order to visit.  Returns
+    (class_of list, n_classes)."""
+    seen, class_of = {}, []
+    for run, segs in segments_by_run:
+        same_class = [Segment(s.run, 0, s.seq, s.n_warps, s.kernel_id, s.records) for s in segs]
+        blob = build(same_class, threads).export()
+        class_of.append(seen.setdefault(blob, len(seen)))
+    return class_of, len(seen)

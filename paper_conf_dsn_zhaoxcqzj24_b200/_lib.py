@@ -38,6 +38,7 @@ SIGNATURES = {
     "owl_adcfg_export": (ctypes.c_int, [vp, ctypes.c_char_p, ctypes.POINTER(vp), ctypes.POINTER(sz)]),
     "owl_adcfg_destroy": (ctypes.c_int, [vp]),
     "owl_diff_adcfg": (ctypes.c_int, [vp, vp, vp, ctypes.POINTER(vp), ctypes.POINTER(sz)]),
+    "owl_filter_inputs": (ctypes.c_int, [vp, ctypes.POINTER(u32), sz, ctypes.POINTER(u32), ctypes.POINTER(u32)]),
     "owl_leak_test": (ctypes.c_int, [vp, vp, vp, ctypes.c_double, ctypes.POINTER(vp), ctypes.POINTER(sz)]),
     "owl_ks_tests": (ctypes.c_int, [vp, vp, vp, ctypes.c_double, ctypes.POINTER(vp), ctypes.POINTER(sz)]),
     "owl_partition_evidence": (ctypes.c_int, [vp, vp, ctypes.c_int, ctypes.POINTER(vp), ctypes.POINTER(u64)]),

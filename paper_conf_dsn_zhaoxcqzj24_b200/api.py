@@ -199,6 +199,16 @@ class Context:
         _check(_lib.load().owl_diff_adcfg(self.h, a.h, b.h, ctypes.byref(p), ctypes.byref(n)))
         return _take(p, n.value, DIFF_DTYPE)
 
+    def filter_inputs(self, runs):
+        """owl_filter_inputs (N1): (class of each run, number of classes); one class <=> the
+        inputs show no trace difference.  Class ids in order of first appearance."""
+        runs = list(runs)
+        arr, n = _u32arr(runs)
+        out = (ctypes.c_uint32 * max(1, n))()
+        nc = ctypes.c_uint32()
+        _check(_lib.load().owl_filter_inputs(self.h, arr, n, out, ctypes.byref(nc)))
+        return np.array(out[:n], dtype=np.uint32), int(nc.value)
+
     def leak_test(self, e_fix: Adcfg, e_rnd: Adcfg, significance: float = 0.05) -> np.ndarray:
         p, n = ctypes.c_void_p(), ctypes.c_size_t()
         _check(_lib.load().owl_leak_test(self.h, e_fix.h, e_rnd.h, significance, ctypes.byref(p), ctypes.byref(n)))

@@ -243,7 +243,9 @@ __device__ __forceinline__ uint32_t dir_hash(uint64_t hi, uint64_t lo) {
   h ^= h >> 13;
   return h;
 }
+#ifndef DIR_PROBES
 #define DIR_PROBES 4
+#endif
 
 /* Admission of a recurring key into the CTA directory (lane 0): claims the first free slot of h ..
    h+DIR_PROBES-1 (the slots lookups probe); a window then gets the next free page.  A key already

@@ -14,6 +14,7 @@
 #include <cstring>
 #include <chrono>
 #include <map>
+#include <memory>
 #include <string>
 #include <tuple>
 #include <vector>
@@ -798,6 +799,62 @@ OWL_API owl_status owl_ks_tests(owl_ctx* ctx, const owl_adcfg* e_fix, const owl_
   if (s != OWL_OK) return s;
   *rows = host_copy(out);
   *n_rows = out.size();
+  return OWL_OK;
+}
+
+/* N1 (§VI): partition runs by identical per-run A-DCFGs.  Fingerprints bucket, exact
+   comparisons with each class's representative decide. */
+OWL_API owl_status owl_filter_inputs(owl_ctx* ctx, const uint32_t* runs, size_t n_runs, uint32_t* class_of,
+                                     uint32_t* n_classes) {
+  if (!ctx || !n_classes || (n_runs && (!runs || !class_of))) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  for (size_t i = 0; i < n_runs; ++i)
+    for (size_t j = 0; j < i; ++j)
+      if (runs[i] == runs[j]) return fail(OWL_ERR_INVALID_ARG, "run %u given twice", runs[i]);
+  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+  struct Rep {
+    std::unique_ptr<owl_adcfg> g;
+    uint32_t cls;
+  };
+  std::map<std::pair<unsigned long long, unsigned long long>, std::vector<Rep>> buckets;
+  uint32_t nc = 0;
+  for (size_t i = 0; i < n_runs; ++i) {
+    owl_adcfg* raw = nullptr;
+    owl_status st = owl_build_adcfg(ctx, &runs[i], 1, &raw);
+    if (st != OWL_OK) return st;
+    std::unique_ptr<owl_adcfg> g(raw);
+    st = ensure_sorted(g.get());
+    if (st != OWL_OK) return st;
+    for (int t = 0; t < T_NUM; ++t) owl_table_free(&g->tab[t]); /* only the sorted cells are compared */
+    unsigned long long fp[2];
+    CUDA_TRY(owl_tables_fingerprint(g->sorted, T_NUM, fp, ctx->stream), "filter: fingerprint");
+    for (uint32_t sl : g->slots.order) { /* the kernel sequence is part of the trace */
+      fp[0] = owl_mix64(fp[0] ^ g->slots.kid[sl]);
+      fp[1] = owl_mix64(fp[1] + g->slots.kid[sl] * 0x9E3779B97F4A7C15ull + g->slots.count[sl]);
+    }
+    std::vector<Rep>& cand = buckets[{fp[0], fp[1]}];
+    int found = -1;
+    for (const Rep& r : cand) {
+      const owl_adcfg* a = r.g.get();
+      bool same = a->slots.order == g->slots.order && a->slots.kid == g->slots.kid && a->slots.count == g->slots.count;
+      if (same) {
+        owl_diff* rows = nullptr;
+        uint64_t nd = 0;
+        CUDA_TRY(owl_diff_rows(a->sorted, g->sorted, T_NUM, &rows, &nd, 0, ctx->stream), "filter: compare");
+        free(rows);
+        same = nd == 0;
+      }
+      if (same) {
+        found = (int)r.cls;
+        break;
+      }
+    }
+    if (found < 0) {
+      found = (int)nc++;
+      cand.push_back(Rep{std::move(g), (uint32_t)found});
+    }
+    class_of[i] = (uint32_t)found;
+  }
+  *n_classes = nc;
   return OWL_OK;
 }
 

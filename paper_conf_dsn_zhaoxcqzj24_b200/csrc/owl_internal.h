@@ -135,6 +135,9 @@ cudaError_t owl_diff_sorted(const SortedTable& a, const SortedTable& b, std::vec
 cudaError_t owl_diff_rows(const SortedTable* A, const SortedTable* B, int ntab, owl_diff** rows, uint64_t* n_rows,
                           size_t extra_rows, cudaStream_t st);
 
+/* order-independent 128-bit fingerprint of the cells of ntab sorted tables (input-class filtering, N1) */
+cudaError_t owl_tables_fingerprint(const SortedTable* tabs, int ntab, unsigned long long fp[2], cudaStream_t st);
+
 /* stable bucketing of a segment's records by gwarp (channel-order input, reading R17) */
 cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, uint4* out, uint64_t* perm,
                                cudaStream_t st);

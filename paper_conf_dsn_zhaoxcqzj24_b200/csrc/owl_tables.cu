@@ -571,6 +571,47 @@ cudaError_t owl_diff_rows(const SortedTable* A, const SortedTable* B, int ntab, 
   return cudaSuccess;
 }
 
+namespace {
+
+__device__ __forceinline__ unsigned long long fmix64(unsigned long long x) {
+  x ^= x >> 33; x *= 0xff51afd7ed558ccdull; x ^= x >> 33; x *= 0xc4ceb9fe1a85ec53ull; x ^= x >> 33;
+  return x;
+}
+
+/* sums (mod 2^64) of two independent mixes of every (table, key, count): equal multisets of cells give
+   equal fingerprints whatever their order */
+__global__ void fingerprint_kernel(const Key128* k, const unsigned long long* c, uint64_t n, int t,
+                                   unsigned long long* fp) {
+  unsigned long long a = 0, b = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long h = fmix64(k[i].hi ^ ((unsigned long long)t << 62)) ^ fmix64(k[i].lo + 0x9E3779B97F4A7C15ull);
+    a += fmix64(h ^ c[i]);
+    b += fmix64(h + c[i] * 0xC2B2AE3D27D4EB4Full + 1);
+  }
+  for (int o = 16; o; o >>= 1) {
+    a += __shfl_xor_sync(0xFFFFFFFFu, a, o);
+    b += __shfl_xor_sync(0xFFFFFFFFu, b, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicAdd(&fp[0], a);
+    atomicAdd(&fp[1], b);
+  }
+}
+
+}  // namespace
+
+cudaError_t owl_tables_fingerprint(const SortedTable* tabs, int ntab, unsigned long long fp[2], cudaStream_t st) {
+  unsigned long long* d = (unsigned long long*)owl_dev_alloc(16);
+  if (!d) return cudaErrorMemoryAllocation;
+  cudaError_t e = cudaMemsetAsync(d, 0, 16, st);
+  for (int t = 0; t < ntab && e == cudaSuccess; ++t)
+    if (tabs[t].n) fingerprint_kernel<<<grid_for(tabs[t].n, 256), 256, 0, st>>>(tabs[t].k, tabs[t].c, tabs[t].n, t, d);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(fp, d, 16, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  owl_dev_free(d);
+  return e;
+}
+
 cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, uint4* out, uint64_t* perm,
                                cudaStream_t st) {
   if (!n) return cudaSuccess;

@@ -336,3 +336,36 @@ def test_wide_keys_sort_fallback(ctx):
     of = oracle.build([oracle.Segment(0, 0, 0, 8, 10, rec)])
     assert _build_one(ctx, rec, 8) == of.export()
     assert H.parse_blob(of.export())["addr"].shape[0] > 4096
+
+
+@pytest.mark.parametrize("cfg,div,nf,nr", [(1, 1, 3, 3), (2, 64, 3, 3), (4, 256, 2, 3), (5, 32, 2, 2)])
+def test_filter_inputs_parity(ctx, cfg, div, nf, nr):
+    """N1: the GPU partition of runs into classes of identical traces equals the oracle's."""
+    p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=nf, runs_rnd=nr)
+    runs = list(range(p.n_runs))
+    ctx.ingest(_gpu_segments(p, runs))
+    try:
+        order = runs[::-1]  # visiting order decides the class ids
+        gc, gn = ctx.filter_inputs(order)
+        by_run = [(r, [oracle.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, tracegen.host_records(p, r, m.seq))
+                       for m in tracegen.run_segments(p, r)]) for r in order]
+        oc, on = oracle.filter_inputs(by_run)
+        assert gn == on and list(gc) == oc
+    finally:
+        ctx.forget_runs(runs)
+
+
+def test_filter_inputs_copies_and_changed_record(ctx):
+    rec = H.w1_records()
+    other = rec.copy()
+    i = int(np.flatnonzero(other["meta"] >> 31)[-1])
+    other["addr"][i] = other["addr"][i] + np.uint64(4)
+    bufs = [torch.from_numpy(x.view(np.uint8).copy()).cuda() for x in (rec, rec, other, rec)]
+    ctx.ingest([api.Segment(r, r % 2, 0, 2, 10, b, len(rec)) for r, b in enumerate(bufs)])
+    try:
+        cls, n = ctx.filter_inputs([0, 1, 2, 3])
+        assert list(cls) == [0, 0, 1, 0] and n == 2
+        with pytest.raises(api.OwlError, match="INVALID_ARG"):
+            ctx.filter_inputs([0, 0])
+    finally:
+        ctx.forget_runs([0, 1, 2, 3])
