@@ -124,6 +124,11 @@ def test_generator_device_equals_host():
                 host = tracegen.host_records(p, r, m.seq)
                 assert n == len(host)
                 assert bytes(buf.cpu().numpy()) == host.tobytes(), (cfg, r, m.seq)
+    for cfg, t in ((6, 1000), (7, 333), (8, 50)):
+        p = tracegen.Params.preset(cfg, threads=t)
+        for m in tracegen.run_segments(p, 0):
+            buf, n = tracegen.device_records(p, 0, m.seq)
+            assert bytes(buf.cpu().numpy()) == tracegen.host_records(p, 0, m.seq).tobytes(), cfg
 
 
 def test_w1(ctx):
@@ -369,3 +374,10 @@ def test_filter_inputs_copies_and_changed_record(ctx):
             ctx.filter_inputs([0, 0])
     finally:
         ctx.forget_runs([0, 1, 2, 3])
+
+
+@pytest.mark.parametrize("cfg,threads", [(6, 100), (6, 3000), (7, 1000), (8, 10)])
+def test_rq2_workloads_parity(ctx, cfg, threads):
+    """N4: the RQ2 trace-size workloads (partial last warps included) fold bit-exactly."""
+    p = tracegen.Params.preset(cfg, threads=threads, runs_fix=1, runs_rnd=1)
+    _build_and_compare(ctx, p)

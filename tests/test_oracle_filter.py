@@ -53,3 +53,30 @@ def test_kernel_sequence_is_part_of_the_trace():
     rec = H.w1_records()
     runs = [(0, [oracle.Segment(0, 0, 0, 2, 10, rec)]), (1, [oracle.Segment(1, 0, 0, 2, 11, rec)])]
     assert oracle.filter_inputs(runs) == ([0, 1], 2)
+
+
+# ---- N4: the RQ2 trace-size workloads (Fig. 5) -------------------------------------------------
+
+def _rq2(cfg, threads):
+    import struct
+    p = tracegen.Params.preset(cfg, threads=threads)
+    segs = [oracle.Segment(0, m.input_class, m.seq, m.n_warps, m.kernel_id, tracegen.host_records(p, 0, m.seq))
+            for m in tracegen.run_segments(p, 0)]
+    blob = oracle.build(segs).export()
+    return sum(len(s.records) for s in segs), struct.unpack_from("<4Q", blob, 24)
+
+
+def test_rq2_growth_patterns():
+    """The three growth patterns of P:L366 as closed forms of the workloads' construction: (1) fixed threads:
+    records and cells constant; (2) S-box lookups: records grow linearly, address cells saturate at 16 x 256;
+    (3) thread-distinct pixels: cells = 5 per thread.  Records = accesses + one BB entry per traced warp."""
+    for t in (100, 777, 4096):
+        warps = -(-t // 32)
+        rec2, cells2 = _rq2(6, t)
+        rec3, cells3 = _rq2(7, t)
+        rec1, cells1 = _rq2(8, t)
+        assert rec2 == 16 * t + warps and cells2[3] <= 16 * 256
+        assert rec3 == 5 * t + warps and cells3[3] == 5 * t
+        assert rec1 == 8 * 256 + 8 and cells1[3] == 64
+        assert cells1[:3] == cells2[:3] == cells3[:3] == (1, 2, 1)  # one BB: node, S->B0, B0->S, one triple
+    assert _rq2(6, 20000)[1][3] == 16 * 256  # saturated

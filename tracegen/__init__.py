@@ -26,13 +26,19 @@ CONFIGS = {
     3: dict(runs_fix=100, runs_rnd=100, grid_div=1),   # RSA modexp, 4K threads
     4: dict(runs_fix=50, runs_rnd=50, grid_div=1),     # PyTorch-shaped ops
     5: dict(runs_fix=500, runs_rnd=500, grid_div=1),   # nvJPEG-shaped decode, 1000 runs
+    # RQ2 trace-size sweep (Fig. 5): threads = the input size
+    6: dict(runs_fix=1, runs_rnd=0, grid_div=1, threads=1024),  # pattern 2: dummy S-box program
+    7: dict(runs_fix=1, runs_rnd=0, grid_div=1, threads=1024),  # pattern 3: thread-distinct pixels
+    8: dict(runs_fix=1, runs_rnd=0, grid_div=1, threads=1024),  # pattern 1: fixed threads
 }
-CONFIG_NAMES = {1: "C1-toy", 2: "C2-aes128-ttable", 3: "C3-rsa-modexp", 4: "C4-pytorch-ops", 5: "C5-nvjpeg-decode"}
+CONFIG_NAMES = {1: "C1-toy", 2: "C2-aes128-ttable", 3: "C3-rsa-modexp", 4: "C4-pytorch-ops", 5: "C5-nvjpeg-decode",
+                6: "RQ2-sbox", 7: "RQ2-pixel", 8: "RQ2-fixed-threads"}
 
 
 class _Params(ctypes.Structure):
     _fields_ = [("config", ctypes.c_uint32), ("grid_div", ctypes.c_uint32), ("runs_fix", ctypes.c_uint32),
-                ("runs_rnd", ctypes.c_uint32), ("seed", ctypes.c_uint64)]
+                ("runs_rnd", ctypes.c_uint32), ("seed", ctypes.c_uint64), ("threads", ctypes.c_uint32),
+                ("_pad", ctypes.c_uint32)]
 
 
 @dataclass(frozen=True)
@@ -42,6 +48,7 @@ class Params:
     runs_rnd: int
     grid_div: int = 1
     seed: int = MASTER_SEED
+    threads: int = 0
 
     @staticmethod
     def preset(config: int, **over) -> "Params":
@@ -50,7 +57,7 @@ class Params:
         return Params(config=config, **kw)
 
     def c(self) -> _Params:
-        return _Params(self.config, self.grid_div, self.runs_fix, self.runs_rnd, self.seed)
+        return _Params(self.config, self.grid_div, self.runs_fix, self.runs_rnd, self.seed, self.threads, 0)
 
     @property
     def n_runs(self) -> int:

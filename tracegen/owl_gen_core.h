@@ -45,11 +45,13 @@ typedef struct {
 } og_record;
 
 typedef struct {
-  uint32_t config;   /* 1..5 */
+  uint32_t config;   /* 1..5 (BASELINE configs), 6..8 (RQ2 sweep) */
   uint32_t grid_div; /* every kernel's block count is divided by this (min 1 block); 1 = paper shape */
   uint32_t runs_fix;
   uint32_t runs_rnd;
   uint64_t seed;     /* master seed; DESIGN.md default 0x4F574C21 */
+  uint32_t threads;  /* configs 6-8 (RQ2 trace-size sweep): the input size = thread count */
+  uint32_t _pad;
 } og_params;
 
 enum { OG_FIX = 0, OG_RND = 1 };
@@ -93,7 +95,8 @@ OG_HD uint32_t og_blocks(const og_params* p, uint32_t dflt) {
 }
 
 /* ---- kernel sequence of a run ------------------------------------------------------------------- */
-enum { OG_K_TOY = 0, OG_K_AES, OG_K_RSA, OG_K_EMBED, OG_K_CONV, OG_K_SOFTMAX, OG_K_NONZERO, OG_K_HUFF, OG_K_IDCT };
+enum { OG_K_TOY = 0, OG_K_AES, OG_K_RSA, OG_K_EMBED, OG_K_CONV, OG_K_SOFTMAX, OG_K_NONZERO, OG_K_HUFF, OG_K_IDCT,
+       OG_K_SBOX, OG_K_PIXEL, OG_K_REPR };
 
 OG_HD int og_c4_allzero(const og_params* p, uint32_t r) {
   return og_run_class(p, r) == OG_RND && (og_h2(og_run_secret(p, r), OG_TAG_ZERO) & 1u);
@@ -112,6 +115,9 @@ OG_HD uint32_t og_seq_kernel(const og_params* p, uint32_t r, uint32_t seq) {
     case 2: return OG_K_AES;
     case 3: return OG_K_RSA;
     case 4: return seq == 0 ? OG_K_EMBED : seq == 1 ? OG_K_CONV : seq == 2 ? OG_K_SOFTMAX : OG_K_NONZERO;
+    case 6: return OG_K_SBOX;
+    case 7: return OG_K_PIXEL;
+    case 8: return OG_K_REPR;
     default: return seq == 0 ? OG_K_HUFF : OG_K_IDCT;
   }
 }
@@ -128,6 +134,9 @@ OG_HD uint32_t og_kernel_blocks(const og_params* p, uint32_t k) {
     case OG_K_SOFTMAX: return og_blocks(p, 256);
     case OG_K_NONZERO: return og_blocks(p, 256);
     case OG_K_HUFF: return og_blocks(p, 32);
+    case OG_K_SBOX:
+    case OG_K_PIXEL: return p->threads ? (p->threads + 255u) / 256u : 1u;
+    case OG_K_REPR: return 1u;
     default: return og_blocks(p, 500); /* IDCT: 500 x 256 = 128,000 threads */
   }
 }
@@ -405,6 +414,39 @@ OG_HD void og_warp_c5(const og_params* p, uint32_t r, uint32_t k, og_em* e) {
   }
 }
 
+/* ---- configs 6-8: the RQ2 trace-size workloads (Fig. 5), input size = p->threads ---------
+   6 (pattern 2, "volatile threads with limited memory accesses"): the paper's dummy program, random
+     lookups into a 256-entry S-box (16 per thread, byte = f(secret, thread, i)); distinct addresses
+     saturate at 16 x 256 while records grow with the threads;
+   7 (pattern 3, "volatile threads with unlimited memory access", nvJPEG-like): every thread loads four
+     words of its own pixel and stores one; distinct addresses grow with the threads;
+   8 (pattern 1, "fixed threads", Tensor.__repr__): one block of 256 threads reads a fixed set of
+     elements whatever the input size.
+   Threads beyond p->threads (the last block's tail) are inactive: they emit nothing. */
+OG_HD void og_warp_rq2(const og_params* p, uint32_t r, uint32_t k, og_em* e) {
+  const uint32_t w = e->gwarp;
+  const uint32_t T = k == OG_K_REPR ? 256u : p->threads;
+  uint32_t l, i;
+  if (w * 32u >= T) return;
+  const uint32_t act = T - w * 32u < 32u ? T - w * 32u : 32u; /* active lanes 0..act-1 */
+  if (k == OG_K_SBOX) {
+    const uint64_t sec = og_run_secret(p, r);
+    og_bb(e, 0);
+    for (i = 0; i < 16; ++i)
+      for (l = 0; l < act; ++l)
+        og_mem(e, l, 0, i, og_addr(OG_T_SHARED, 1, 4ull * (og_h3(sec, w * 32 + l, i) & 0xFFu)));
+  } else if (k == OG_K_PIXEL) {
+    og_bb(e, 0);
+    for (i = 0; i < 4; ++i)
+      for (l = 0; l < act; ++l) og_mem(e, l, 0, i, og_addr(OG_T_GLOBAL, 2, 16ull * (w * 32 + l) + 4 * i));
+    for (l = 0; l < act; ++l) og_mem(e, l, 0, 4, og_addr(OG_T_GLOBAL, 3, 4ull * (w * 32 + l)));
+  } else {
+    og_bb(e, 0);
+    for (i = 0; i < 8; ++i)
+      for (l = 0; l < act; ++l) og_mem(e, l, 0, i, og_addr(OG_T_GLOBAL, 4, 4ull * (((w * 32 + l) * 8 + i) & 63u)));
+  }
+}
+
 /* Records of traced warp `gwarp` of invocation `seq` of run `r`, in program order; returns the count.
    out == NULL counts only. */
 OG_HD uint64_t og_warp(const og_params* p, uint32_t r, uint32_t seq, uint32_t gwarp, og_record* out) {
@@ -418,6 +460,7 @@ OG_HD uint64_t og_warp(const og_params* p, uint32_t r, uint32_t seq, uint32_t gw
     case 2: og_warp_c2(p, r, &e); break;
     case 3: og_warp_c3(p, r, &e); break;
     case 4: og_warp_c4(p, r, k, &e); break;
+    case 6: case 7: case 8: og_warp_rq2(p, r, k, &e); break;
     default: og_warp_c5(p, r, k, &e); break;
   }
   return e.n;
