@@ -189,16 +189,17 @@ def count_launches(step):
     return sum(names.values()), names
 
 
-def e2e_leg(args, p, api, tracegen, dev, stream, n_runs_e2e):
+def e2e_leg(args, p, api, tracegen, dev, stream, n_runs_e2e, my_runs, world=1, rank=0):
     """Same metric through the public C ABI with HOST records: every step stages the runs' records from
-    pinned host memory into HBM inside owl_build_adcfg (OWL_SEG_HOST_RECORDS), folds, diffs and runs the
-    leak test, whose rows come back to the host (D2H).  A subset of the workload's runs (stated) keeps the
-    pinned host footprint bounded."""
+    pinned host memory into HBM inside owl_build_adcfg (OWL_SEG_HOST_RECORDS), folds, (at N > 1 exchanges
+    cells by owner,) diffs and runs the leak test, whose rows come back to the host (D2H).  The first
+    n_runs_e2e of each rank's runs (stated) keep the pinned host footprint bounded."""
     import torch
+    import torch.distributed as dist
     ctx = api.Context(dev.index)
     base_run = 1 << 20  # run ids disjoint from the device-resident leg
-    runs_f = [r for r in range(p.n_runs) if tracegen.run_class(p, r) == 0][: n_runs_e2e // 2]
-    runs_r = [r for r in range(p.n_runs) if tracegen.run_class(p, r) == 1][: n_runs_e2e // 2]
+    runs_f = [r for r in my_runs if tracegen.run_class(p, r) == 0][: n_runs_e2e // 2]
+    runs_r = [r for r in my_runs if tracegen.run_class(p, r) == 1][: n_runs_e2e // 2]
     segs, hold, n_rec = [], [], 0
     for r in runs_f + runs_r:
         for m in tracegen.run_segments(p, r):
@@ -214,18 +215,34 @@ def e2e_leg(args, p, api, tracegen, dev, stream, n_runs_e2e):
     ctx.ingest(segs, stream)
     rf = [base_run + r for r in runs_f]
     rr = [base_run + r for r in runs_r]
+    if world > 1:
+        from paper_conf_dsn_zhaoxcqzj24_b200 import dist as D
+        mine = rf + rr
+        meta = {base_run + r: (tracegen.run_class(p, r), [m.kernel_id for m in tracegen.run_segments(p, r)])
+                for r in runs_f + runs_r}
+        allm = D.gather_sequences(meta)
+        D.agree_slots(ctx, allm, mine)
+        rf = sorted(r for r, (c, _) in allm.items() if c == 0)
+        rr = sorted(r for r, (c, _) in allm.items() if c == 1)
     d2h = [0]
 
     def step():
         ef, er = ctx.build(rf), ctx.build(rr)
-        d = ctx.diff(ef, er)
-        lk = ctx.leak_test(ef, er, 0.05)
+        held = [ef, er]
+        if world > 1:
+            (ef, bf), (er, br) = D.owner_evidence(ctx, ef, world, rank), D.owner_evidence(ctx, er, world, rank)
+            held += [ef, er]
+            d, lk = D.diff(ctx, ef, er), D.leak_test(ctx, ef, er, 0.05)
+        else:
+            d, lk = ctx.diff(ef, er), ctx.leak_test(ef, er, 0.05)
         d2h[0] = d.nbytes + lk.nbytes
-        ef.destroy()
-        er.destroy()
+        for g in held:
+            g.destroy()
 
     for _ in range(max(1, args.warmup)):
         step()
+    if world > 1:
+        dist.barrier()
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     steps = max(1, min(args.steps, 3))
@@ -235,11 +252,18 @@ def e2e_leg(args, p, api, tracegen, dev, stream, n_runs_e2e):
     e1.record(stream)
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / steps
+    total = n_rec
+    if world > 1:
+        t = torch.tensor([ms, float(n_rec)], device=dev, dtype=torch.float64)
+        mx = t.clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        ms, total = float(mx[0].item()), int(t[1].item())
     del ctx, segs, hold
-    return {"value": n_rec / (ms / 1e3), "unit": "records/s", "h2d_bytes_per_step": 16 * n_rec,
-            "d2h_bytes_per_step": d2h[0], "ms_per_step": ms, "records_per_step": n_rec,
-            "sample": f"{len(rf)} FIX + {len(rr)} RND runs of the same workload from pinned host memory, "
-                      f"{steps} steps"}
+    return {"value": total / (ms / 1e3), "unit": "records/s", "h2d_bytes_per_step": 16 * total,
+            "d2h_bytes_per_step": d2h[0], "ms_per_step": ms, "records_per_step": total,
+            "sample": f"{len(runs_f)} FIX + {len(runs_r)} RND runs per GPU of the same workload from pinned host "
+                      f"memory, {steps} steps"}
 
 
 def run_ours(args):
@@ -250,8 +274,16 @@ def run_ours(args):
     from paper_conf_dsn_zhaoxcqzj24_b200 import api
 
     world, rank, local = _dist()
+    # OWL_BENCH_SHARE_GPU=1 (tests only): ranks share the box's GPUs round-robin and use gloo, so the N > 1
+    # path can be exercised on one GPU; the measured configuration is one rank per GPU over NCCL.
+    share = os.environ.get("OWL_BENCH_SHARE_GPU") == "1"
+    if share:
+        local = local % torch.cuda.device_count()
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     cfg = args.config
@@ -274,7 +306,18 @@ def run_ours(args):
     t_gen = time.perf_counter() - t_gen
     n_records = sum(s.n_records for s in segs)
     ctx.ingest(segs, stream)
-    rf, rr = _class_runs(p, my_runs, 0), _class_runs(p, my_runs, 1)
+    all_runs = list(range(p.n_runs))
+    if world > 1:
+        # §8(e): slot agreement over all runs, then every step folds this rank's shard into partial evidences
+        # and exchanges cells by owner (paper_conf_dsn_zhaoxcqzj24_b200/dist.py)
+        from paper_conf_dsn_zhaoxcqzj24_b200 import dist as D
+        meta = {r: (tracegen.run_class(p, r), [m.kernel_id for m in tracegen.run_segments(p, r)]) for r in my_runs}
+        all_meta = D.gather_sequences(meta)
+        D.agree_slots(ctx, all_meta, my_runs)
+        all_runs = sorted(all_meta)
+        rf, rr = _class_runs(p, all_runs, 0), _class_runs(p, all_runs, 1)
+    else:
+        rf, rr = _class_runs(p, my_runs, 0), _class_runs(p, my_runs, 1)
 
     out = {}
     brk = {}
@@ -293,13 +336,22 @@ def run_ours(args):
         t0 = tick("build_fix", t0)
         er = ctx.build(rr)
         t0 = tick("build_rnd", t0)
-        d = ctx.diff(ef, er)
-        t0 = tick("diff", t0)
-        lk = ctx.leak_test(ef, er, 0.05)
+        held = [ef, er]
+        if world > 1:  # the one exchange: partial evidences -> owners' evidences
+            (ef, bf), (er, br) = D.owner_evidence(ctx, ef, world, rank), D.owner_evidence(ctx, er, world, rank)
+            held += [ef, er]
+            t0 = tick("exchange", t0)
+            d = D.diff(ctx, ef, er)
+            t0 = tick("diff", t0)
+            lk = D.leak_test(ctx, ef, er, 0.05)
+        else:
+            d = ctx.diff(ef, er)
+            t0 = tick("diff", t0)
+            lk = ctx.leak_test(ef, er, 0.05)
         t0 = tick("leak_test", t0)
         out.update(n_diff=len(d), n_leaks=len(lk), info_f=ef.info(), info_r=er.info())
-        ef.destroy()
-        er.destroy()
+        for g in held:
+            g.destroy()
         tick("destroy", t0)
 
     clocks = ClockSampler(local)
@@ -358,7 +410,7 @@ def run_ours(args):
         del segs
         ctx.forget_runs(my_runs)
         torch.cuda.empty_cache()
-        res["e2e"] = e2e_leg(args, p, api, tracegen, dev, stream, args.e2e_runs)
+        res["e2e"] = e2e_leg(args, p, api, tracegen, dev, stream, args.e2e_runs, my_runs, world, rank)
     if rank == 0 and not args.no_cpu:
         res["cpu_baseline"] = cpu_baseline(cfg, args.cpu_seconds)
     if rank == 0:

@@ -381,3 +381,56 @@ def test_rq2_workloads_parity(ctx, cfg, threads):
     """N4: the RQ2 trace-size workloads (partial last warps included) fold bit-exactly."""
     p = tracegen.Params.preset(cfg, threads=threads, runs_fix=1, runs_rnd=1)
     _build_and_compare(ctx, p)
+
+
+@pytest.mark.parametrize("cfg,div,nf,nr", [(2, 64, 3, 3), (4, 256, 2, 3)])
+def test_sharded_exchange_equals_one_gpu(cfg, div, nf, nr):
+    """§8(e) on one GPU: two 'ranks' (two contexts) each fold a shard of the runs with agreed slots, partition
+    their partial evidences by owner, the buckets are exchanged (the all-to-all, done by hand), and each owner
+    absorbs its cells: the owners' leak rows, KS rows and diff rows, merged, equal the oracle's on all runs."""
+    from paper_conf_dsn_zhaoxcqzj24_b200 import dist as D
+    p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=nf, runs_rnd=nr)
+    runs = list(range(p.n_runs))
+    world = 2
+    ctxs = [api.Context(0) for _ in range(world)]
+    keep = []
+    meta = {r: (tracegen.run_class(p, r), [m.kernel_id for m in tracegen.run_segments(p, r)]) for r in runs}
+    parts = {}
+    for rank, c in enumerate(ctxs):
+        mine = D.shard(runs, world, rank)
+        segs = _gpu_segments(p, mine)
+        keep.append(segs)
+        c.ingest(segs)
+        D.agree_slots(c, meta, mine)
+        for cls in (0, 1):
+            parts[(rank, cls)] = c.build([r for r in runs if tracegen.run_class(p, r) == cls])
+    owned = {}
+    for cls in (0, 1):
+        bufs = []
+        for rank in range(world):
+            ptr, sb = parts[(rank, cls)].partition(world)
+            whole = torch.as_tensor(D._DeviceBytes(ptr, sum(sb)), device="cuda") if sum(sb) else \
+                torch.empty(0, dtype=torch.uint8, device="cuda")
+            bufs.append((whole.clone(), sb))
+        for owner in range(world):
+            pieces, rb = [], []
+            for rank in range(world):
+                whole, sb = bufs[rank]
+                off = sum(sb[:owner])
+                pieces.append(whole[off: off + sb[owner]])
+                rb.append(sb[owner])
+            recv = torch.cat(pieces)
+            keep.append(recv)
+            owned[(owner, cls)] = ctxs[owner].absorb(parts[(owner, cls)], recv.data_ptr() if recv.numel() else None,
+                                                     rb, owner)
+    leaks = D.merge_leaks([ctxs[o].leak_test(owned[(o, 0)], owned[(o, 1)], SIG) for o in range(world)])
+    diffs = D.merge_diffs([ctxs[o].diff(owned[(o, 0)], owned[(o, 1)]) for o in range(world)])
+    ks = np.concatenate([ctxs[o].ks_tests(owned[(o, 0)], owned[(o, 1)], SIG) for o in range(world)])
+    osg = _oracle_segments(p, runs)
+    of, orr = oracle.build(osg[0]), oracle.build(osg[1])
+    assert_leak_parity(leaks, oracle.leak_test(of, orr, SIG))
+    od = oracle.diff(of, orr)
+    assert len(diffs) == len(od) and np.array_equal(diffs, od)
+    oks = oracle.ks_tests(of, orr, SIG)
+    key = lambda a: np.lexsort((a["j"], a["ins"], a["bb"], a["slot_fix"], a["kind"]))  # noqa: E731
+    assert_ks_parity(ks[key(ks)], oks[key(oks)])
