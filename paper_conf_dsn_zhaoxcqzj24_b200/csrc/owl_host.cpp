@@ -217,7 +217,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
                      uint64_t* n_records) {
   const cudaStream_t st = ctx->stream;
   *overflow = 0;
-  const uint32_t tile_shift = getenv("OWL_TILE_SHIFT") ? (uint32_t)atoi(getenv("OWL_TILE_SHIFT")) : 14u;
+  const uint32_t tile_shift = getenv("OWL_TILE_SHIFT") ? (uint32_t)atoi(getenv("OWL_TILE_SHIFT")) : 15u; /* tile sweep: profiles/r01_v4_ab.txt */
   std::vector<FoldSeg> fs(plan.size());
   std::vector<void*> scratch;
   std::vector<uint64_t*> perms(plan.size(), nullptr);
