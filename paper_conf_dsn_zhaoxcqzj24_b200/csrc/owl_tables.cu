@@ -158,9 +158,12 @@ __global__ void gather_diff_kernel(const uint64_t* idx, const unsigned long long
   }
 }
 
-__global__ void bucket_keys_kernel(const uint4* rec, uint64_t n, uint32_t* gw, uint64_t* idx) {
+/* key = gwarp, with every out-of-range gwarp mapped to n_warps (a stable sort keeps their relative order;
+   the fold reports the first of them): the sort needs only ceil(log2(n_warps + 1)) bits */
+__global__ void bucket_keys_kernel(const uint4* rec, uint64_t n, uint32_t n_warps, uint32_t* gw, uint64_t* idx) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    gw[i] = rec[i].z;
+    const uint32_t g = rec[i].z;
+    gw[i] = g < n_warps ? g : n_warps;
     idx[i] = i;
   }
 }
@@ -621,10 +624,9 @@ cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, u
   cudaError_t e = (gw && gw2 && idx) ? cudaSuccess : cudaErrorMemoryAllocation;
   void* dt = nullptr;
   if (e == cudaSuccess) {
-    bucket_keys_kernel<<<grid_for(n, 256), 256, 0, st>>>(rec, n, gw, idx);
+    bucket_keys_kernel<<<grid_for(n, 256), 256, 0, st>>>(rec, n, n_warps, gw, idx);
     int bits = 1;
-    while (bits < 32 && (1ull << bits) <= (uint64_t)n_warps) ++bits; /* gwarp >= n_warps sorts last (bit 31) */
-    bits = 32;  /* records with out-of-range gwarp must keep their relative order too */
+    while (bits < 32 && (1ull << bits) <= (uint64_t)n_warps) ++bits; /* keys 0..n_warps */
     size_t tmp = 0;
     cub::DeviceRadixSort::SortPairs(nullptr, tmp, gw, gw2, idx, perm, (int64_t)n, 0, bits, st);
     dt = owl_dev_alloc(tmp);
