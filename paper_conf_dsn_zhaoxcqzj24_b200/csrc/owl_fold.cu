@@ -2,31 +2,30 @@
  * owl_fold.cu — A1-A3: stream trace records once and fold them thread -> warp -> kernel into the
  * A-DCFG hash tables (§V.A-B).
  *
- * Design v7 (measurements in profiles/): the fold is an HBM stream whose per-record work
- * must fit the issue budget (≈5.5 warp-instructions per record at 50% of HBM on 148 SMs), so every choice
- * below minimises instructions per 32-record chunk:
+ * Design v12 (every variant and its measurement in profiles/r01_v4_ab.txt): the fold is an
+ * HBM stream whose per-record work must fit the issue budget, and at 24 warps per SM the register budget
+ * (80) binds, so every choice below minimises instructions per 32-record chunk and live registers:
  *
- *  * persistent CTAs of FOLD_WARPS independent warps; a warp pops one work item (segment, tile of 2^k
+ *  * persistent CTAs of FOLD_WARPS independent warps; a warp pops one work item (segment, tile of 2^15
  *    records) at a time from a global counter.  A tile holds the traced warps whose first record lies in
  *    it: the warp finds the first such start with a 33-ary warp-cooperative search and finishes the last
  *    traced warp past the tile end;
  *  * a warp walks its traced warp FOLD_U chunks of 32 records at a time (one 128-bit streaming load per
  *    lane and chunk), with cp.async.bulk.prefetch.L2 keeping the next granules of its stream in flight;
- *  * A2: a chunk whose 32 records are well-formed MEM records of the current basic block takes the fast
- *    path (its context (cur, j) is warp-uniform).  A chunk holding a BB_ENTRY, a warp end or a malformed
- *    record takes the slow path: it consumes records up to its last BB_ENTRY, applies the entries in lane
- *    order with warp-uniform state (cur, prev, the per-warp visit ordinal j of each BB in a shared-memory
- *    map), counts node / edge / triple cells in a shared-memory table, and gives every MEM lane
- *    the context of the last BB_ENTRY lane before it.  The next chunk then starts on an instruction
- *    boundary, so a fast chunk is normally one instruction executed by 32 threads;
- *  * A3, "merging identical thread traces" before any global atomic.  A fast chunk is
- *      - broadcast (32 equal keys): one add of 32 to its cell in the CTA's shared-memory directory;
- *      - page-local (one attribute, one 1 KB window of addresses, 4-byte aligned — T-table lookups,
- *        tiles of shared memory): each lane adds 1 to a keyless 4-byte bin of the window's shared-memory
- *        page (pages are admitted on a window's second sighting while they last);
- *      - otherwise (thread-distinct addresses, pages exhausted, slow-chunk lanes): one insert per lane
- *        into the global open-addressing table, first probes of all chunks of the step in flight
- *        together, counts added with fire-and-forget RED.64 in L2.
+ *  * A2: a chunk of 32 well-formed MEM records of the current basic block is the fast path (context
+ *    warp-uniform).  A BB_ENTRY in lane 0 (chunks start on instruction boundaries) is consumed alone,
+ *    inline: node / edge / triple cells go to per-kind shared tables (three lanes), the visit ordinal j
+ *     comes from a visit map held in registers (lane l: one BB and its count; more than 32 BBs
+ *    spill to a per-warp map in global scratch), and the rest of the step is realigned with a funnel
+ *    shift across lanes instead of a reload.  Anything else (several entries, warp end, malformed
+ *    records) takes the generic noinline slow path, which mirrors the oracle walk;
+ *  * A3, "merging identical thread traces" before any global atomic: a broadcast chunk (32
+ *    equal keys) is one add of 32; every lane then looks its key up on its own in the CTA directory
+ *    (hot broadcast cells hold their count there; a hot 1 KB address window of one attribute owns a page
+ *    of keyless 4-byte bins and the lane adds 1 to its bin).  Keys enter the directory on their 16th
+ *    sighting (4-way bucketed filter), so one-off windows never take pages.  Lanes that miss insert into
+ *    the global open-addressing table: first probes of the step's chunks in flight together, counts added
+ *    with fire-and-forget RED.64 in L2.
  *    The shared directory / pages / CF cells are exact partial sums, flushed to the global tables when
  *    the CTA finishes.
  * Malformed records are reported with the minimum (segment, index) and skipped (state unaffected),
