@@ -707,10 +707,13 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
                 }
               }
             }
-            /* a key not in the directory: count a sighting, admit recurring keys */
+            /* a key not in the directory: count a sighting, admit recurring keys (one vote skips it all
+               for the usual chunk, whose lanes all hit) */
+            const bool miss = !f && (!bc || lane == 0);
+            if (__any_sync(FULL, miss)) {
             bool ready = false;
             uint32_t fi = 0;
-            if (!f && (!bc || lane == 0)) {
+            if (miss) {
               STAT(2);
               /* 4-way filter bucket: the key's entry, else the entry with the fewest sightings is replaced
                  (hot keys sharing a bucket do not evict each other); racy updates: counts are approximate */
@@ -733,6 +736,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
               ready = (ne & 0xFFu) >= ADMIT;
             }
             if (__any_sync(FULL, ready)) admit_ready(s, ready, khi[u], lo, h0, fi, !bc, lane);
+            }
           }
         } else if (__shfl_sync(FULL, r.z == w.g0 && (r.w & 0xFC0000FFu) == 0 && r.x == 0 && r.y == 0, 0) &&
                    !(w.st & W_SKIP) && FOLD_MODE_OF(a) == 0) {
