@@ -652,7 +652,6 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
       bool lead[FOLD_U];
       uint32_t cnt[FOLD_U];
       uint64_t khi[FOLD_U], klo[FOLD_U];
-      unsigned any_lead = 0;
       bool stop = false; /* the traced warp ended inside the step: the rest is reloaded */
 #pragma unroll
       for (int u = 0; u < FOLD_U; ++u) {
@@ -779,10 +778,11 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
             for (int c = FOLD_U - 1; c > u; --c) rr[c] = funnel(rr[c - 1], rr[c], k, lane);
           }
         }
-        any_lead |= __ballot_sync(FULL, lead[u]);
-
       }
-      if (!any_lead || FOLD_MODE_OF(a) == 1) continue;
+      bool mine = false; /* one vote per step: does any lane of any chunk go to the global table? */
+#pragma unroll
+      for (int u = 0; u < FOLD_U; ++u) mine = mine || lead[u];
+      if (!__any_sync(FULL, mine) || FOLD_MODE_OF(a) == 1) continue;
       /* global table: first probes of all chunks in flight together, predicated REDs, rare misses */
       uint32_t home[FOLD_U];
       ulonglong4 kk[FOLD_U];
