@@ -791,7 +791,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         home[u] = tab_index(khi[u], klo[u], shift);
         kk[u] = ld_bucket_keys_if(lead[u], tab_b + (home[u] >> 1));
       }
-      unsigned miss_any = 0;
+      bool missed = false;
 #pragma unroll
       for (int u = 0; u < FOLD_U; ++u) {
         const bool h0 = kk[u].x == khi[u] && kk[u].y == klo[u];
@@ -799,9 +799,9 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         const bool hit = lead[u] && (h0 || h1);
         red_add_if(hit, &tab_b[home[u] >> 1].count[h1 ? 1 : 0], cnt[u]);
         lead[u] = lead[u] && !hit; /* now: missed (absent, or displaced past the home bucket) */
-        miss_any |= __ballot_sync(FULL, lead[u]);
+        missed = missed || lead[u];
       }
-      if (miss_any) {
+      if (__any_sync(FULL, missed)) {
 #pragma unroll
         for (int u = 0; u < FOLD_U; ++u)
           if (lead[u]) claims += addr_insert_slow(a.tab[T_ADDR], home[u], khi[u], klo[u], cnt[u], a.status);
