@@ -235,9 +235,12 @@ __device__ __noinline__ void cf_insert(FoldSmem& s, const FoldArgs& a, int tbl, 
 
 /* 32-bit mixed hash of a directory key: top DIR_LOG bits = home slot, low FILTER_LOG bits = filter slot */
 __device__ __forceinline__ uint32_t dir_hash(uint64_t hi, uint64_t lo) {
-  uint32_t h = ((uint32_t)hi * 0x9E3779B1u) ^ ((uint32_t)(hi >> 32) * 0x85EBCA77u) ^ ((uint32_t)lo * 0xC2B2AE3Du) ^
-               ((uint32_t)(lo >> 32) * 0x27D4EB2Fu);
-  h ^= h >> 15; /* the keys of one program differ in few low bits (ins, j, window): finish the mixing */
+  /* the keys of one program differ in few low bits (ins, j, window): a sum of multiplicative hashes of the
+     four 32-bit words, then a finishing mix (xor-shift, multiply, xor-shift) so the top bits (home slot)
+     depend on all of them */
+  uint32_t h = (uint32_t)hi + (uint32_t)(hi >> 32) * 0x9E3779B1u + (uint32_t)lo * 0x85EBCA77u +
+               (uint32_t)(lo >> 32) * 0xC2B2AE3Du;
+  h ^= h >> 16;
   h *= 0x2C1B3C6Du;
   h ^= h >> 13;
   return h;
