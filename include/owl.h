@@ -100,7 +100,18 @@ typedef struct {
   uint32_t max_regrow;      /* times a build may double a full table and re-run (default 6)       */
   uint32_t fold_ctas_per_sm;/* 0 = automatic                                                      */
   uint64_t host_chunk_bytes;/* staging chunk for OWL_SEG_HOST_RECORDS (0 = 256 MiB)               */
+  uint32_t hcf_reading;     /* y-values of H_cf (SURVEY reading 5): OWL_HCF_COUNTS (0,
+                               default) = joint counts c_ij; OWL_HCF_ROW_NORMALIZED (1) = the elements
+                               a_ij = c_ij / x_i of the transition matrix A (Eqs. 7-8).  Other values:
+                               OWL_ERR_INVALID_ARG from owl_ctx_set_config.                          */
+  uint32_t _reserved;
 } owl_config;
+
+/* H_cf readings.  R2 weights each (src, dst) cell of a node by a_ij = c_ij / x_i, with
+   x_i = sum_j c_ij the src count of Eq. 5, and tests F(t) = sum_{cells <= t} a / k (k = number of srcs,
+   the sum of all a_ij) on both sides; D is fp64 (not an exact integer ratio), the KS row's K_lo = K_hi
+   = 0, and n, m remain the node counts of Eq. 5. */
+enum { OWL_HCF_COUNTS = 0, OWL_HCF_ROW_NORMALIZED = 1 };
 
 /* Tables of an A-DCFG (§V.B).  Canonical key order in brackets. */
 enum {

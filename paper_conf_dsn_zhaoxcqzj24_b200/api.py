@@ -151,8 +151,11 @@ class Context:
                 pass
             self.h = None
 
-    def set_config(self, addr_capacity=0, cf_capacity=0, max_regrow=0, fold_ctas_per_sm=0, host_chunk_bytes=0):
-        cfg = _lib.OwlConfig(addr_capacity, cf_capacity, max_regrow, fold_ctas_per_sm, host_chunk_bytes)
+    def set_config(self, addr_capacity=0, cf_capacity=0, max_regrow=0, fold_ctas_per_sm=0, host_chunk_bytes=0,
+                   hcf_reading=0):
+        """owl_ctx_set_config.  hcf_reading: 0 = joint counts (R1), 1 = row-normalized A (R2, Eq. 7)."""
+        cfg = _lib.OwlConfig(addr_capacity, cf_capacity, max_regrow, fold_ctas_per_sm, host_chunk_bytes,
+                             hcf_reading, 0)
         _check(_lib.load().owl_ctx_set_config(self.h, ctypes.byref(cfg)))
 
     def ingest(self, segments, stream=None):

@@ -514,6 +514,8 @@ OWL_API owl_status owl_ctx_destroy(owl_ctx* ctx) {
 
 OWL_API owl_status owl_ctx_set_config(owl_ctx* ctx, const owl_config* cfg) {
   if (!ctx) return fail(OWL_ERR_INVALID_ARG, "ctx is NULL");
+  if (cfg && cfg->hcf_reading > OWL_HCF_ROW_NORMALIZED)
+    return fail(OWL_ERR_INVALID_ARG, "hcf_reading must be OWL_HCF_COUNTS or OWL_HCF_ROW_NORMALIZED");
   if (cfg) ctx->cfg = *cfg;
   else ctx->cfg = owl_config{};
   for (int t = 0; t < T_NUM; ++t) ctx->cap_hint[t] = 0;
@@ -758,7 +760,8 @@ owl_status run_ks(owl_ctx* ctx, const owl_adcfg* f, const owl_adcfg* r, double s
   std::vector<std::tuple<int, uint32_t, uint32_t, uint32_t, uint32_t, size_t>> order;
   for (int tbl : {T_TRIPLE, T_ADDR}) {
     std::vector<KsOutRow> out;
-    CUDA_TRY(owl_ks_run(tbl, f->sorted[tbl], r->sorted[tbl], al.f2r, sig, out, ctx->stream), "KS tests");
+    CUDA_TRY(owl_ks_run(tbl, f->sorted[tbl], r->sorted[tbl], al.f2r, sig, (int)ctx->cfg.hcf_reading, out,
+                        ctx->stream), "KS tests");
     for (const KsOutRow& o : out) {
       owl_ks_row row;
       Key128 kf{o.hi_f, 0}, kr{o.hi_r, 0};

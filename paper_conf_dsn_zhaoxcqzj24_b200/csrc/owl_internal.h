@@ -150,7 +150,7 @@ struct KsOutRow {
   uint32_t fail, _pad;
 };
 cudaError_t owl_ks_run(int tbl, const SortedTable& f, const SortedTable& r, const std::vector<uint32_t>& slot_f2r,
-                       double significance, std::vector<KsOutRow>& rows, cudaStream_t st);
+                       double significance, int hcf_reading, std::vector<KsOutRow>& rows, cudaStream_t st);
 
 /* multi-GPU: pack every cell of the four sorted tables by owner rank */
 struct ExchangeCell {

@@ -169,6 +169,94 @@ __device__ double u128_to_double_rn(u128 v) {
   return scalbn((double)mant, e);
 }
 
+/* ---- H_cf reading R2 (Eqs. 5-8) --------------------------------------------
+ * The node's cells (prev, next) are weighted by a_ij = c_ij / x_i (x_i = the row's total, Eq. 5, so that
+ * I.A = O, Eq. 7) and H = (a_11, ..., a_kp) (Eq. 8) is tested as a weighted sample: F(t) = sum_{cells<=t} a / k
+ * with k = number of rows (= sum of all a).  Cells are row-major, so at a union position t = (p, q) a side's
+ * F is (rows before p + cum_p(q) / x_p) / k when it has row p, else (rows before p) / k: one division per
+ * side and position, in this fixed order.  One thread per attribute pair walks the two sorted lists (nodes
+ * hold at most a few hundred cells; this is latency-bound, not a roofline kernel). */
+struct R2State {
+  uint64_t i, e;
+  uint32_t rows, cur;
+  bool have;
+  unsigned long long cum, x;
+};
+
+__device__ __forceinline__ uint32_t prev_of(const Key128& k) { return (uint32_t)(k.lo >> 32); }
+
+__device__ uint32_t r2_rows(const Key128* k, uint64_t b, uint64_t e) {
+  uint32_t r = 0;
+  for (uint64_t i = b; i < e; ++i) r += (i == b || prev_of(k[i]) != prev_of(k[i - 1])) ? 1u : 0u;
+  return r;
+}
+
+__device__ void r2_step(const Key128* k, const unsigned long long* c, R2State& s, unsigned long long t) {
+  if (s.i >= s.e || k[s.i].lo != t) return;
+  const uint32_t p = (uint32_t)(t >> 32);
+  if (!s.have || p != s.cur) {
+    if (s.have) ++s.rows;
+    s.have = true;
+    s.cur = p;
+    s.cum = 0;
+    s.x = 0;
+    for (uint64_t i = s.i; i < s.e && prev_of(k[i]) == p; ++i) s.x += c[i];
+  }
+  s.cum += c[s.i];
+  ++s.i;
+}
+
+__device__ double r2_F(const R2State& s, uint32_t tp, double kd) {
+  if (!s.have) return 0.0;
+  if (s.cur == tp)
+    return __ddiv_rn(__dadd_rn(__uint2double_rn(s.rows), __ddiv_rn(__ull2double_rn(s.cum), __ull2double_rn(s.x))),
+                     kd);
+  return __ddiv_rn(__uint2double_rn(s.rows + 1u), kd); /* its row before tp is complete */
+}
+
+__device__ __forceinline__ void ks_p_value(unsigned long long n, unsigned long long m, double D, double significance,
+                                           double& pv, uint32_t& fail) {
+  const double nd = __ull2double_rn(n), md = __ull2double_rn(m);
+  const double nm = __dmul_rn(nd, md);
+  const double wgt = __ddiv_rn(nm, __dadd_rn(nd, md));
+  const double x = __dmul_rn(__dmul_rn(2.0, __dmul_rn(D, D)), wgt);
+  pv = __dmul_rn(2.0, exp(-x));
+  fail = pv < significance ? 1u : 0u;
+}
+
+__global__ void ks_r2_kernel(const Key128* fk, const unsigned long long* fc, const unsigned long long* fpre, uint64_t nf,
+                             const uint64_t* stf, uint64_t naf, const Key128* rk, const unsigned long long* rc,
+                             const unsigned long long* rpre, uint64_t nr, const uint64_t* str, uint64_t nar,
+                             const uint2* pairs, uint64_t np, double significance, KsOutRow* out) {
+  for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < np; p += (uint64_t)gridDim.x * blockDim.x) {
+    const Range r = range_of(pairs[p], stf, naf, nf, str, nar, nr);
+    const unsigned long long n = fpre[r.fe - 1], m = rpre[r.re - 1];
+    const double kf = __uint2double_rn(r2_rows(fk, r.fb, r.fe)), kr = __uint2double_rn(r2_rows(rk, r.rb, r.re));
+    R2State a{r.fb, r.fe, 0u, 0u, false, 0ull, 0ull}, b{r.rb, r.re, 0u, 0u, false, 0ull, 0ull};
+    double D = 0.0;
+    while (a.i < a.e || b.i < b.e) {
+      const unsigned long long t =
+          (a.i < a.e && (b.i >= b.e || fk[a.i].lo <= rk[b.i].lo)) ? fk[a.i].lo : rk[b.i].lo;
+      r2_step(fk, fc, a, t);
+      r2_step(rk, rc, b, t);
+      const uint32_t tp = (uint32_t)(t >> 32);
+      const double d = fabs(__dsub_rn(r2_F(a, tp, kf), r2_F(b, tp, kr)));
+      if (d > D) D = d;
+    }
+    KsOutRow o;
+    o.hi_f = fk[r.fb].hi;
+    o.hi_r = rk[r.rb].hi;
+    o.n = n;
+    o.m = m;
+    o.K_lo = 0;
+    o.K_hi = 0;
+    o.D = D;
+    ks_p_value(n, m, D, significance, o.p, o.fail);
+    o._pad = 0;
+    out[p] = o;
+  }
+}
+
 __global__ void ks_final_kernel(const Key128* fk, const unsigned long long* fpre, uint64_t nf, const uint64_t* stf,
                                 uint64_t naf, const Key128* rk, const unsigned long long* rpre, uint64_t nr,
                                 const uint64_t* str, uint64_t nar, const uint2* pairs, uint64_t np,
@@ -248,7 +336,7 @@ cudaError_t prepare(const SortedTable& t, Side& s, cudaStream_t st) {
 }  // namespace
 
 cudaError_t owl_ks_run(int tbl, const SortedTable& f, const SortedTable& r, const std::vector<uint32_t>& slot_f2r,
-                       double significance, std::vector<KsOutRow>& rows, cudaStream_t st) {
+                       double significance, int hcf_reading, std::vector<KsOutRow>& rows, cudaStream_t st) {
   rows.clear();
   if (!f.n || !r.n || slot_f2r.empty()) return cudaSuccess;
   Side sf, sr;
@@ -275,7 +363,17 @@ cudaError_t owl_ks_run(int tbl, const SortedTable& f, const SortedTable& r, cons
     e = cudaMemcpyAsync(&np, npairs, 8, cudaMemcpyDeviceToHost, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   }
-  if (e == cudaSuccess && np) {
+  if (e == cudaSuccess && np && tbl == T_TRIPLE && hcf_reading == OWL_HCF_ROW_NORMALIZED) {
+    dout = (KsOutRow*)owl_dev_alloc(np * sizeof(KsOutRow));
+    if (!dout) e = cudaErrorMemoryAllocation;
+    if (e == cudaSuccess) {
+      ks_r2_kernel<<<grid_for(np, 128), 128, 0, st>>>(f.k, f.c, sf.pre, f.n, sf.starts, sf.na, r.k, r.c, sr.pre, r.n,
+                                                      sr.starts, sr.na, pairs, np, significance, dout);
+      rows.resize(np);
+      e = cudaMemcpyAsync(rows.data(), dout, np * sizeof(KsOutRow), cudaMemcpyDeviceToHost, st);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    }
+  } else if (e == cudaSuccess && np) {
     nunits = (unsigned long long*)owl_dev_alloc(np * 8);
     uoff = (unsigned long long*)owl_dev_alloc((np + 1) * 8);
     dout = (KsOutRow*)owl_dev_alloc(np * sizeof(KsOutRow));

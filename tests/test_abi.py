@@ -64,3 +64,20 @@ def test_oracle_shares_no_header_with_product():
     src = open(os.path.join(ROOT, "oracle", "owl_oracle.cpp")).read()
     includes = re.findall(r'#include\s+[<"]([^>"]+)[>"]', src)
     assert all("/" not in i and not i.startswith("owl") for i in includes), includes
+
+
+def test_binding_layouts_match_header(tmp_path):
+    """The ctypes structs and numpy row dtypes of the binding have the header's sizes and field offsets."""
+    import subprocess
+    from paper_conf_dsn_zhaoxcqzj24_b200 import _lib, api
+    c = tmp_path / "sz.c"
+    c.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "owl.h"\nint main(void){printf("%zu %zu %zu %zu %zu '
+                 '%zu %zu %zu\\n", sizeof(owl_config), offsetof(owl_config, hcf_reading), sizeof(owl_segment), '
+                 'sizeof(owl_adcfg_info), sizeof(owl_diff), sizeof(owl_leak), sizeof(owl_ks_row), '
+                 'offsetof(owl_ks_row, D));return 0;}\n')
+    exe = tmp_path / "sz"
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), str(c), "-o", str(exe)], check=True)
+    got = [int(v) for v in subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split()]
+    assert got == [ctypes.sizeof(_lib.OwlConfig), _lib.OwlConfig.hcf_reading.offset, ctypes.sizeof(_lib.OwlSegment),
+                   ctypes.sizeof(_lib.OwlAdcfgInfo), api.DIFF_DTYPE.itemsize, api.LEAK_DTYPE.itemsize,
+                   api.KS_DTYPE.itemsize, api.KS_DTYPE.fields["D"][1]]

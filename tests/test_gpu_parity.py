@@ -434,3 +434,72 @@ def test_sharded_exchange_equals_one_gpu(cfg, div, nf, nr):
     oks = oracle.ks_tests(of, orr, SIG)
     key = lambda a: np.lexsort((a["j"], a["ins"], a["bb"], a["slot_fix"], a["kind"]))  # noqa: E731
     assert_ks_parity(ks[key(ks)], oks[key(oks)])
+
+
+# ---- N3: H_cf reading R2 (row-normalized transition matrix A, Eqs. 7-8) -------------------------------
+def _r2_oracle_rows(of, orr, o_ks):
+    """R2 statistic for every CF pair the oracle tests (same pairs as R1: node present on both aligned sides)."""
+    from oracle import hcf_r2
+    tf, tr = H.parse_blob(of.export())["triple"], H.parse_blob(orr.export())["triple"]
+    out = []
+    for row in o_ks[o_ks["kind"] == 1]:
+        cf = hcf_r2.node_cells(tf, int(row["slot_fix"]), int(row["bb"]))
+        cr = hcf_r2.node_cells(tr, int(row["slot_rnd"]), int(row["bb"]))
+        out.append(hcf_r2.ks_r2(cf, cr, SIG))
+    return out
+
+
+@pytest.mark.parametrize("cfg,div,nf,nr", [(1, 1, 10, 10), (2, 32, 3, 3), (3, 16, 2, 2), (4, 64, 2, 2)])
+def test_hcf_r2_parity(ctx, cfg, div, nf, nr):
+    """Bar for R2: n, m exact; K = 0; |D - D_exact| <= 1e-12 (D is a rational evaluated in fp64
+    on the GPU, exactly on the oracle); p within the band that D tolerance implies through Eq. 4
+    (|dp/p| <= 4 D w |dD| + 1e-12); verdicts identical outside that band; DF rows identical to R1's."""
+    p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=nf, runs_rnd=nr)
+    runs = list(range(p.n_runs))
+    ctx.ingest(_gpu_segments(p, runs))
+    try:
+        ef, er = ctx.build(_runs_of(p, 0)), ctx.build(_runs_of(p, 1))
+        osg = _oracle_segments(p, runs)
+        of, orr = oracle.build(osg[0]), oracle.build(osg[1])
+        o_ks = oracle.ks_tests(of, orr, SIG)
+        ctx.set_config(hcf_reading=1)
+        try:
+            g_ks = ctx.ks_tests(ef, er, SIG)
+            g_leaks = ctx.leak_test(ef, er, SIG)
+        finally:
+            ctx.set_config()
+        assert len(g_ks) == len(o_ks)
+        for f in ("kind", "slot_fix", "slot_rnd", "bb", "ins", "j", "n", "m"):
+            assert np.array_equal(g_ks[f], o_ks[f]), f
+        df = g_ks["kind"] == 2
+        assert_ks_parity(g_ks[df], o_ks[df])
+        cf = np.flatnonzero(g_ks["kind"] == 1)
+        r2 = _r2_oracle_rows(of, orr, o_ks)
+        assert len(r2) == len(cf) and len(cf) > 0
+        fails = set()
+        for i, (n, m, D, Dd, po, fo) in zip(cf, r2):
+            g = g_ks[i]
+            assert int(g["K_lo"]) == 0 and int(g["K_hi"]) == 0
+            Dg = float(g["D"])
+            assert abs(Dg - float(D)) <= 1e-12, (i, Dg, D)
+            w = n * m / (n + m)
+            band = 4.0 * Dd * w * 1e-12 + 1e-12
+            pg = float(g["p"])
+            assert abs(pg - po) <= band * max(po, pg) or (po == 0.0 and pg < 1e-300), (i, pg, po)
+            if bool(g["fail"]) != fo:
+                assert abs(po - SIG) <= band * SIG, (i, pg, po)
+            if g["fail"]:
+                fails.add((int(g["slot_fix"]), int(g["bb"])))
+        g_cf = {(int(r["slot_fix"]), int(r["bb"])) for r in g_leaks if r["kind"] == 1}
+        assert g_cf == fails
+        o_leaks = oracle.leak_test(of, orr, SIG)
+        keep_g, keep_o = g_leaks["kind"] != 1, o_leaks["kind"] != 1  # kernel / DF leaks: independent of H_cf
+        assert_leak_parity(g_leaks[keep_g], o_leaks[keep_o])
+    finally:
+        ctx.forget_runs(runs)
+
+
+def test_hcf_reading_invalid(ctx):
+    with pytest.raises(api.OwlError, match="OWL_ERR_INVALID_ARG"):
+        ctx.set_config(hcf_reading=2)
+    ctx.set_config()
