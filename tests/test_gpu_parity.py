@@ -434,6 +434,14 @@ def test_sharded_exchange_equals_one_gpu(cfg, div, nf, nr):
     oks = oracle.ks_tests(of, orr, SIG)
     key = lambda a: np.lexsort((a["j"], a["ins"], a["bb"], a["slot_fix"], a["kind"]))  # noqa: E731
     assert_ks_parity(ks[key(ks)], oks[key(oks)])
+    for c in ctxs:  # owners test their own nodes under R2 as well (each node's cells live on one owner)
+        c.set_config(hcf_reading=1)
+    ks2 = np.concatenate([ctxs[o].ks_tests(owned[(o, 0)], owned[(o, 1)], SIG) for o in range(world)])
+    ks2 = ks2[key(ks2)]
+    oks = oks[key(oks)]
+    for f in ("kind", "slot_fix", "slot_rnd", "bb", "ins", "j", "n", "m"):
+        assert np.array_equal(ks2[f], oks[f]), f
+    _assert_r2_rows(ks2, oks, of, orr)
 
 
 # ---- N3: H_cf reading R2 (row-normalized transition matrix A, Eqs. 7-8) -------------------------------
@@ -449,7 +457,31 @@ def _r2_oracle_rows(of, orr, o_ks):
     return out
 
 
-@pytest.mark.parametrize("cfg,div,nf,nr", [(1, 1, 10, 10), (2, 32, 3, 3), (3, 16, 2, 2), (4, 64, 2, 2)])
+def _assert_r2_rows(g_ks, o_ks, of, orr):
+    """GPU KS rows under R2 (same order as the oracle's R1 rows) against the rational R2 oracle; returns the
+    (slot_fix, bb) of the failing CF rows."""
+    cf = np.flatnonzero(g_ks["kind"] == 1)
+    r2 = _r2_oracle_rows(of, orr, o_ks)
+    assert len(r2) == len(cf) and len(cf) > 0
+    fails = set()
+    for i, (n, m, D, Dd, po, fo) in zip(cf, r2):
+        g = g_ks[i]
+        assert int(g["K_lo"]) == 0 and int(g["K_hi"]) == 0
+        Dg = float(g["D"])
+        assert abs(Dg - float(D)) <= 1e-12, (i, Dg, D)
+        w = n * m / (n + m)
+        band = 4.0 * Dd * w * 1e-12 + 1e-12
+        pg = float(g["p"])
+        assert abs(pg - po) <= band * max(po, pg) or (po == 0.0 and pg < 1e-300), (i, pg, po)
+        if bool(g["fail"]) != fo:
+            assert abs(po - SIG) <= band * SIG, (i, pg, po)
+        if g["fail"]:
+            fails.add((int(g["slot_fix"]), int(g["bb"])))
+    return fails
+
+
+@pytest.mark.parametrize("cfg,div,nf,nr", [(1, 1, 10, 10), (2, 32, 3, 3), (3, 16, 2, 2), (4, 64, 2, 2),
+                                        (5, 16, 3, 3)])
 def test_hcf_r2_parity(ctx, cfg, div, nf, nr):
     """Bar for R2: n, m exact; K = 0; |D - D_exact| <= 1e-12 (D is a rational evaluated in fp64
     on the GPU, exactly on the oracle); p within the band that D tolerance implies through Eq. 4
@@ -473,23 +505,7 @@ def test_hcf_r2_parity(ctx, cfg, div, nf, nr):
             assert np.array_equal(g_ks[f], o_ks[f]), f
         df = g_ks["kind"] == 2
         assert_ks_parity(g_ks[df], o_ks[df])
-        cf = np.flatnonzero(g_ks["kind"] == 1)
-        r2 = _r2_oracle_rows(of, orr, o_ks)
-        assert len(r2) == len(cf) and len(cf) > 0
-        fails = set()
-        for i, (n, m, D, Dd, po, fo) in zip(cf, r2):
-            g = g_ks[i]
-            assert int(g["K_lo"]) == 0 and int(g["K_hi"]) == 0
-            Dg = float(g["D"])
-            assert abs(Dg - float(D)) <= 1e-12, (i, Dg, D)
-            w = n * m / (n + m)
-            band = 4.0 * Dd * w * 1e-12 + 1e-12
-            pg = float(g["p"])
-            assert abs(pg - po) <= band * max(po, pg) or (po == 0.0 and pg < 1e-300), (i, pg, po)
-            if bool(g["fail"]) != fo:
-                assert abs(po - SIG) <= band * SIG, (i, pg, po)
-            if g["fail"]:
-                fails.add((int(g["slot_fix"]), int(g["bb"])))
+        fails = _assert_r2_rows(g_ks, o_ks, of, orr)
         g_cf = {(int(r["slot_fix"]), int(r["bb"])) for r in g_leaks if r["kind"] == 1}
         assert g_cf == fails
         o_leaks = oracle.leak_test(of, orr, SIG)
