@@ -226,8 +226,9 @@ owl_status owl_ks_tests(owl_ctx* ctx, const owl_adcfg* e_fix, const owl_adcfg* e
 
 /* ---- multi-GPU (the collective is issued by the caller through torch.distributed / NCCL) ----------
  * owl_partition_evidence packs every cell of a partial evidence into `world` contiguous device buckets
- * by owner(attr) = mix64(attr) mod world, attr = (slot,bb) for node/edge-by-src/triple cells and
- * (slot,bb,ins,j) for address cells.  *d_send is a device buffer owned by the adcfg (valid until it is
+ * by owner(attr) = mix64(attr) mod world, attr = bb for node/edge-by-src/triple cells and (bb,ins,j)
+ * for address cells (no slot: both sides of an aligned fix/rnd slot pair meet on one rank whatever
+ * their slot ids).  *d_send is a device buffer owned by the adcfg (valid until it is
  * destroyed); send_bytes[world] receives the bucket sizes (bytes, multiple of 32).
  * owl_absorb_evidence sums received buckets (laid out back to back in d_recv, recv_bytes[world]) into
  * a new evidence `owned` holding exactly the attributes this rank owns.  Slot ids must agree across
@@ -236,6 +237,18 @@ owl_status owl_partition_evidence(owl_ctx* ctx, const owl_adcfg* partial, int wo
                                   uint64_t* send_bytes);
 owl_status owl_absorb_evidence(owl_ctx* ctx, const owl_adcfg* like, const void* d_recv, const uint64_t* recv_bytes,
                                int world, int rank, owl_adcfg** owned);
+/* Merge of the owners' result rows into the one-GPU result.  parts: the concatenation
+ * of every owner's owl_leak_test rows (any order).  e_fix / e_rnd: this rank's evidences (any of them: the
+ * slot tables are replicated).  Output, as owl_leak_test on one GPU: the kernel-leak rows (recomputed from
+ * the slot tables), then CF rows, then DF rows, each by (alignment position, bb, ins); a DF location
+ * whose visits j were tested on several owners keeps its min-p row, ties -> smallest j (reading
+ * R14).  Errors: INVALID_ARG for a NULL argument or a row whose fix slot is not aligned in e_fix. */
+owl_status owl_merge_leaks(owl_ctx* ctx, const owl_adcfg* e_fix, const owl_adcfg* e_rnd, const owl_leak* parts,
+                           size_t n_parts, owl_leak** leaks, size_t* n_leaks);
+/* Same for owl_diff_adcfg rows: the owners' table rows (disjoint) in canonical (table, key) order, then the
+ * slot rows recomputed from a's and b's slot tables.  INVALID_ARG for a NULL argument or a bad table id. */
+owl_status owl_merge_diffs(owl_ctx* ctx, const owl_adcfg* a, const owl_adcfg* b, const owl_diff* parts,
+                           size_t n_parts, owl_diff** rows, size_t* n_rows);
 /* Registers the kernel sequences of runs this rank does not hold (gathered from the other ranks) so
  * that Myers slot assignment (A4) sees every run of the class in global order. kernel_ids is the
  * concatenation of the runs' sequences; seq_len[i] is run i's length. */

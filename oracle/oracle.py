@@ -37,20 +37,25 @@ _lib = None
 def lib():
     global _lib
     if _lib is None:
-        L = ctypes.CDLL(os.path.join(_HERE, "liboracle.so"))
-        vp, sz = ctypes.c_void_p, ctypes.c_size_t
-        L.orc_build.argtypes = [ctypes.POINTER(_Seg), sz, ctypes.c_int]; L.orc_build.restype = vp
-        L.orc_free.argtypes = [vp]; L.orc_free.restype = None
-        L.orc_last_error.restype = ctypes.c_char_p
-        L.orc_export.argtypes = [vp, vp, sz]; L.orc_export.restype = sz
-        L.orc_diff.argtypes = [vp, vp, vp, sz]; L.orc_diff.restype = sz
-        L.orc_ks_tests.argtypes = [vp, vp, ctypes.c_double, vp, sz]; L.orc_ks_tests.restype = sz
-        L.orc_leak_test.argtypes = [vp, vp, ctypes.c_double, vp, sz]; L.orc_leak_test.restype = sz
-        L.orc_myers.argtypes = [vp, sz, vp, sz, vp, sz]; L.orc_myers.restype = sz
-        L.orc_ks_hist.argtypes = [vp, vp, sz, vp, vp, sz, ctypes.c_double, vp]; L.orc_ks_hist.restype = None
-        L.orc_slots.argtypes = [vp, vp, vp, vp, sz]; L.orc_slots.restype = sz
-        _lib = L
+        _lib = bind(ctypes.CDLL(os.path.join(_HERE, "liboracle.so")))
     return _lib
+
+
+def bind(L):
+    """Declares the C signatures on a loaded oracle library (also used by the mutation tests, which load
+    deliberately broken builds of owl_oracle.cpp to show that the pins catch them)."""
+    vp, sz = ctypes.c_void_p, ctypes.c_size_t
+    L.orc_build.argtypes = [ctypes.POINTER(_Seg), sz, ctypes.c_int]; L.orc_build.restype = vp
+    L.orc_free.argtypes = [vp]; L.orc_free.restype = None
+    L.orc_last_error.restype = ctypes.c_char_p
+    L.orc_export.argtypes = [vp, vp, sz]; L.orc_export.restype = sz
+    L.orc_diff.argtypes = [vp, vp, vp, sz]; L.orc_diff.restype = sz
+    L.orc_ks_tests.argtypes = [vp, vp, ctypes.c_double, vp, sz]; L.orc_ks_tests.restype = sz
+    L.orc_leak_test.argtypes = [vp, vp, ctypes.c_double, vp, sz]; L.orc_leak_test.restype = sz
+    L.orc_myers.argtypes = [vp, sz, vp, sz, vp, sz]; L.orc_myers.restype = sz
+    L.orc_ks_hist.argtypes = [vp, vp, sz, vp, vp, sz, ctypes.c_double, vp]; L.orc_ks_hist.restype = None
+    L.orc_slots.argtypes = [vp, vp, vp, vp, sz]; L.orc_slots.restype = sz
+    return L
 
 
 class OracleError(RuntimeError):

@@ -44,6 +44,8 @@ SIGNATURES = {
     "owl_partition_evidence": (ctypes.c_int, [vp, vp, ctypes.c_int, ctypes.POINTER(vp), ctypes.POINTER(u64)]),
     "owl_absorb_evidence": (ctypes.c_int, [vp, vp, vp, ctypes.POINTER(u64), ctypes.c_int, ctypes.c_int,
                                            ctypes.POINTER(vp)]),
+    "owl_merge_leaks": (ctypes.c_int, [vp, vp, vp, vp, sz, ctypes.POINTER(vp), ctypes.POINTER(sz)]),
+    "owl_merge_diffs": (ctypes.c_int, [vp, vp, vp, vp, sz, ctypes.POINTER(vp), ctypes.POINTER(sz)]),
     "owl_register_remote_runs": (ctypes.c_int, [vp, ctypes.POINTER(u32), ctypes.POINTER(u32), ctypes.POINTER(u32),
                                                 ctypes.POINTER(u64), sz]),
     "owl_get_stats": (ctypes.c_int, [vp, ctypes.POINTER(u64), ctypes.POINTER(ctypes.c_double), ctypes.POINTER(u64),

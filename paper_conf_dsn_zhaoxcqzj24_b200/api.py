@@ -222,6 +222,24 @@ class Context:
         _check(_lib.load().owl_ks_tests(self.h, e_fix.h, e_rnd.h, significance, ctypes.byref(p), ctypes.byref(n)))
         return _take(p, n.value, KS_DTYPE)
 
+    def merge_leaks(self, e_fix: Adcfg, e_rnd: Adcfg, parts) -> np.ndarray:
+        """owl_merge_leaks: the owners' leak rows (list of arrays) -> the one-GPU leak list."""
+        rows = np.ascontiguousarray(np.concatenate(list(parts)) if len(parts) else np.zeros(0, LEAK_DTYPE),
+                                    dtype=LEAK_DTYPE)
+        p, n = ctypes.c_void_p(), ctypes.c_size_t()
+        _check(_lib.load().owl_merge_leaks(self.h, e_fix.h, e_rnd.h, rows.ctypes.data if len(rows) else None,
+                                           len(rows), ctypes.byref(p), ctypes.byref(n)))
+        return _take(p, n.value, LEAK_DTYPE)
+
+    def merge_diffs(self, a: Adcfg, b: Adcfg, parts) -> np.ndarray:
+        """owl_merge_diffs: the owners' diff rows (list of arrays) -> canonical order, slot rows once."""
+        rows = np.ascontiguousarray(np.concatenate(list(parts)) if len(parts) else np.zeros(0, DIFF_DTYPE),
+                                    dtype=DIFF_DTYPE)
+        p, n = ctypes.c_void_p(), ctypes.c_size_t()
+        _check(_lib.load().owl_merge_diffs(self.h, a.h, b.h, rows.ctypes.data if len(rows) else None, len(rows),
+                                           ctypes.byref(p), ctypes.byref(n)))
+        return _take(p, n.value, DIFF_DTYPE)
+
     def absorb(self, like: Adcfg, recv_ptr, recv_bytes, rank) -> Adcfg:
         world = len(recv_bytes)
         rb = (ctypes.c_uint64 * world)(*recv_bytes)

@@ -1,8 +1,9 @@
 /*
  * owl_exchange.cu — the one data exchange of the multi-GPU path: every cell of
- * a rank's partial evidence goes to owner(attr) = mix64(key_hi) mod world.  key_hi is (slot, bb) for node,
- * edge-by-src and triple cells and (slot, bb, ins, j) for address cells, so all cells of one KS attribute
- * (a node's H_cf, an instruction-visit's H_addr) meet on one rank.  The payload is exchanged by the caller
+ * a rank's partial evidence goes to owner(attr) = mix64(attr) mod world, attr = bb for node, edge-by-src and
+ * triple cells and (bb, ins, j) for address cells (the slot is left out: fix and rnd slots of one aligned
+ * pair may differ), so all cells of one KS attribute (a node's H_cf, an instruction-visit's H_addr) of
+ * both evidences meet on one rank.  The payload is exchanged by the caller
  * with torch.distributed all_to_all_single (NCCL over NVLink); the owner sums it into its tables (integer
  * sums: bit-identical to one GPU).
  */
@@ -15,21 +16,25 @@ using namespace owl_dev;
 
 namespace {
 
-__device__ __forceinline__ uint32_t owner_of(unsigned long long hi, int world) {
-  unsigned long long x = hi;
+/* owner of a cell: a hash of its attribute WITHOUT the slot field.  The two evidences number their slots
+   independently and the KS pairs fix slot s with rnd slot f2r[s] (owl_ks.cu), so both sides of one attribute
+   must meet on one rank whatever their slot ids: (bb) for node / edge-by-src / triple cells, (bb, ins, j)
+   for address cells (owl_internal.h key layout). */
+__device__ __forceinline__ uint32_t owner_of(unsigned long long hi, int tbl, int world) {
+  unsigned long long x = tbl == T_ADDR ? (hi & ((1ull << 48) - 1)) : (hi & 0xFFFFFFFFull);
   x ^= x >> 33; x *= 0xff51afd7ed558ccdull; x ^= x >> 33; x *= 0xc4ceb9fe1a85ec53ull; x ^= x >> 33;
   return (uint32_t)(x % (unsigned long long)world);
 }
 
-__global__ void count_owner_kernel(const Key128* k, uint64_t n, int world, unsigned long long* counts) {
+__global__ void count_owner_kernel(const Key128* k, uint64_t n, int tbl, int world, unsigned long long* counts) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
-    atomicAdd(&counts[owner_of(k[i].hi, world)], 1ull);
+    atomicAdd(&counts[owner_of(k[i].hi, tbl, world)], 1ull);
 }
 
 __global__ void scatter_owner_kernel(const Key128* k, const unsigned long long* c, uint64_t n, int tbl, int world,
                                      const unsigned long long* offs, unsigned long long* cursor, ExchangeCell* out) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t o = owner_of(k[i].hi, world);
+    const uint32_t o = owner_of(k[i].hi, tbl, world);
     const unsigned long long pos = offs[o] + atomicAdd(&cursor[o], 1ull);
     ExchangeCell e;
     e.hi = k[i].hi;
@@ -74,7 +79,7 @@ cudaError_t owl_partition_cells(const SortedTable* tabs, int world, ExchangeCell
   cudaMemsetAsync(dcnt, 0, world * 8, st);
   cudaMemsetAsync(dcur, 0, world * 8, st);
   for (int t = 0; t < T_NUM; ++t)
-    if (tabs[t].n) count_owner_kernel<<<grid_for(tabs[t].n, 256), 256, 0, st>>>(tabs[t].k, tabs[t].n, world, dcnt);
+    if (tabs[t].n) count_owner_kernel<<<grid_for(tabs[t].n, 256), 256, 0, st>>>(tabs[t].k, tabs[t].n, t, world, dcnt);
   std::vector<unsigned long long> h(world), off(world);
   cudaError_t e = cudaMemcpyAsync(h.data(), dcnt, world * 8, cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);

@@ -106,6 +106,8 @@ struct RunDesc {
   uint32_t gen;          /* generation of the traced warp in the overflow visit map */
   const uint4* p_acc;    /* records walked since the last accounting start here */
   uint32_t* seen;
+  unsigned long long* seg_walked; /* records walked in this segment (all CTAs): must end = n */
+  const unsigned long long* perm; /* bucketed segment: caller's index of each record, else NULL */
   uint32_t slot, n_warps, seg_index;
 };
 
@@ -274,8 +276,11 @@ __device__ __noinline__ int dir_admit(FoldSmem& s, uint64_t hi, uint64_t lo, uin
   return 0;
 }
 
-__device__ __forceinline__ void report(FoldStatus* st, uint32_t seg_index, uint64_t idx, uint32_t code) {
-  atomicMin(&st->first_error, ((unsigned long long)seg_index << 40) | (idx << 3) | code);
+/* a malformed record: the minimum (segment, index in the caller's order) wins, as in the oracle; records
+   of a bucketed (channel-order) segment are mapped back through its permutation */
+__device__ __noinline__ void report(FoldStatus* st, const RunDesc& d, uint64_t idx, uint32_t code) {
+  if (d.perm) idx = d.perm[idx];
+  atomicMin(&st->first_error, ((unsigned long long)d.seg_index << 40) | (idx << 3) | code);
 }
 
 /* visits[b] += 1 in the warp's map; returns the new visit ordinal j (reading R8).  Entries of
@@ -310,18 +315,23 @@ __device__ __forceinline__ uint32_t visits_inc(uint32_t* vk, uint32_t* vc, uint3
   return 1;
 }
 
-/* First traced-warp start in [b, e), or e if the tile begins inside a traced warp running past e. */
+/* First traced-warp start in [b, e), or e if the tile begins inside a traced warp running past e.  Valid
+   for warp-major segments, where the records equal to rec[b-1].z form one run; samples that contradict
+   that (a different gwarp before a sample equal to it) end the search at b: the walk then starts inside a
+   traced warp it shares with the previous tile, and the duplicate-warp / walked-record checks report the
+   segment as not warp-major (never a hang, never a silently skipped record). */
 __device__ __forceinline__ uint64_t first_warp_start(const uint4* rec, uint64_t b, uint64_t e, int lane) {
   if (b == 0) return 0;
   const uint32_t gp = __ldg(&rec[b - 1].z);
   if (__ldg(&rec[b].z) != gp) return b;
   if (__ldg(&rec[e - 1].z) == gp) return e;
-  uint64_t lo = b, hi = e - 1; /* rec[lo] == gp, rec[hi] != gp */
+  uint64_t lo = b, hi = e - 1; /* rec[lo] == gp, rec[hi] != gp, lo < hi */
   while (hi - lo > 1) {
-    const uint64_t p = lo + ((hi - lo) * (uint64_t)(lane + 1)) / 33u;
+    const uint64_t p = lo + ((hi - lo) * (uint64_t)(lane + 1)) / 33u; /* ascending in lane */
     const bool same = (p <= lo) ? true : (p >= hi ? false : (__ldg(&rec[p].z) == gp));
     const unsigned m = __ballot_sync(FULL, same);
     const unsigned nm = ~m;
+    if (m && nm && 31 - __clz(m) > __ffs(nm) - 1) return b; /* not one contiguous run: not warp-major */
     const uint64_t plo = __shfl_sync(FULL, p, m ? 31 - __clz(m) : 0);
     const uint64_t phi = __shfl_sync(FULL, p, nm ? __ffs(nm) - 1 : 0);
     if (m && plo > lo) lo = plo;
@@ -408,7 +418,7 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
   if (!(w.st & W_SKIP)) {
     const bool isbb = active && (meta >> 31) == 0;
     const bool bbbad = isbb && (addr != 0 || (meta & 0x7C0000FFu) != 0);
-    if (bbbad) report(a.status, d.seg_index, idx, KERR_BBFIELDS);
+    if (bbbad) report(a.status, d, idx, KERR_BBFIELDS);
     const unsigned bbmask = __ballot_sync(FULL, isbb && !bbbad);
     const uint32_t cur0 = w.cur, j0 = d.curj;
     uint32_t myj = 0;
@@ -454,7 +464,7 @@ __device__ __noinline__ SlowRes slow_chunk(const uint4 r, const unsigned vm, Wal
       if ((addr >> 60) > 8) code = KERR_MTYPE;
       else if (cbb == OWL_NONE_BB) code = KERR_NOBB;
       else if (bbf != cbb) code = KERR_BBMISMATCH;
-      if (code) report(a.status, d.seg_index, idx, code);
+      if (code) report(a.status, d, idx, code);
     }
     good = ismem && code == 0;
     if (good && cj > OWL_MAX_J) atomicOr(&a.status->limit, 1u);
@@ -484,7 +494,7 @@ __device__ __forceinline__ void begin_traced_warp(Walker& w, RunDesc& d, const F
   w.g0 = __ldg(&w.p->z);
   w.st = W_INWARP;
   if (w.g0 >= d.n_warps) { /* every record of this warp is malformed (the first one is reported) */
-    if (lane == 0) report(a.status, d.seg_index, (uint64_t)(w.p - d.rec), KERR_GWARP);
+    if (lane == 0) report(a.status, d, (uint64_t)(w.p - d.rec), KERR_GWARP);
     w.st |= W_SKIP;
   } else if (lane == 0) {
     const uint32_t bit = 1u << (w.g0 & 31);
@@ -592,6 +602,8 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     if (lane == 0) {
       d.rec = sg.rec;
       d.seen = sg.seen;
+      d.seg_walked = sg.walked;
+      d.perm = sg.perm;
       d.slot = sg.slot;
       d.n_warps = sg.n_warps;
       d.seg_index = sg.seg_index;
@@ -629,6 +641,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         if (lane == 0) {
           const unsigned long long n = (unsigned long long)(w.p - d.p_acc);
           if (atomicAdd(&s.walked, n) + n > SHARED_TOTAL_LIMIT) s.off = 1;
+          atomicAdd(d.seg_walked, n);
           d.p_acc = w.p;
         }
         __syncwarp();
@@ -824,6 +837,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     if (lane == 0) {
       const unsigned long long n = (unsigned long long)(w.p - d.p_acc);
       if (atomicAdd(&s.walked, n) + n > SHARED_TOTAL_LIMIT) s.off = 1;
+      if (n) atomicAdd(d.seg_walked, n);
     }
     /* cells claimed by this item -> table fill; past the load limit the build stops and regrows */
     if (__any_sync(FULL, claims != 0)) {

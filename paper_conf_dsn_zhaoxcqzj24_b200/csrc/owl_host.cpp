@@ -227,6 +227,10 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
   if (!seen) return fail(OWL_ERR_OUT_OF_MEMORY, "fold: warp bitmap");
   scratch.push_back(seen);
   CUDA_TRY(cudaMemsetAsync(seen, 0, (seen_words + 1) * 4, st), "fold: memset");
+  unsigned long long* walked = (unsigned long long*)owl_dev_alloc((plan.size() + 1) * 8);
+  if (!walked) { owl_dev_free(seen); return fail(OWL_ERR_OUT_OF_MEMORY, "fold: walk counters"); }
+  scratch.push_back(walked);
+  CUDA_TRY(cudaMemsetAsync(walked, 0, (plan.size() + 1) * 8, st), "fold: memset");
   uint64_t so = 0;
   owl_status status = OWL_OK;
   for (size_t i = 0; i < plan.size() && status == OWL_OK; ++i) {
@@ -257,6 +261,8 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     fs[i].slot = plan[i].slot;
     fs[i].n_warps = s.n_warps;
     fs[i].seen = seen + so;
+    fs[i].walked = walked + i;
+    fs[i].perm = (const unsigned long long*)perms[i];
     fs[i].seg_index = (uint32_t)i;
     fs[i]._pad = 0;
     so += (s.n_warps + 31) / 32;
@@ -296,6 +302,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     if (!dsegs || !dgroups) status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: segment table");
   }
   FoldStatus hs;
+  std::vector<unsigned long long> walked_h(plan.size(), 0);
   if (status == OWL_OK) {
     scratch.push_back(dsegs);
     scratch.push_back(dgroups);
@@ -326,6 +333,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     cudaError_t e = !a.vmap ? cudaErrorMemoryAllocation : items ? owl_launch_fold(a, grid, st) : cudaSuccess;
     cudaEventRecord(ctx->ev1, st);
     if (e == cudaSuccess) e = cudaMemcpyAsync(&hs, ctx->d_status, sizeof hs, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(walked_h.data(), walked, plan.size() * 8, cudaMemcpyDeviceToHost, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     if (e != cudaSuccess) status = cuda_fail(e, "fold kernel");
     else {
@@ -348,13 +356,9 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
   if (status == OWL_OK) {
     if (hs.first_error != ~0ull) {
       const uint32_t si = (uint32_t)(hs.first_error >> 40);
-      uint64_t idx = (hs.first_error >> 3) & ((1ull << 37) - 1);
+      const uint64_t idx = (hs.first_error >> 3) & ((1ull << 37) - 1); /* caller's index (the fold maps
+                                                                           bucketed records back) */
       const uint32_t code = (uint32_t)(hs.first_error & 7);
-      if (si < plan.size() && perms[si]) { /* map back to the caller's record index */
-        uint64_t orig = idx;
-        cudaMemcpy(&orig, perms[si] + idx, 8, cudaMemcpyDeviceToHost);
-        idx = orig;
-      }
       status = fail(OWL_ERR_MALFORMED_TRACE, "malformed trace: run %u seq %u record %llu: %s",
                     si < plan.size() ? plan[si].s.run : 0, si < plan.size() ? plan[si].s.seq : 0,
                     (unsigned long long)idx, kerr_text(code));
@@ -363,6 +367,18 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
       status = fail(OWL_ERR_INVALID_ARG,
                     "segment (run %u, seq %u) is flagged OWL_SEG_WARP_MAJOR but warp %u's records are not contiguous",
                     plan[si].s.run, plan[si].s.seq, (uint32_t)hs.not_warp_major);
+    } else if (!hs.overflow && [&] {
+                 for (size_t i = 0; i < plan.size(); ++i)
+                   if (walked_h[i] != plan[i].s.n_records) return true;
+                 return false;
+               }()) {
+      size_t si = 0;
+      while (walked_h[si] == plan[si].s.n_records) ++si;
+      status = fail(OWL_ERR_INVALID_ARG,
+                    "segment (run %u, seq %u) is flagged OWL_SEG_WARP_MAJOR but its records are not grouped by warp "
+                    "(the warp walk covered %llu records of %llu)",
+                    plan[si].s.run, plan[si].s.seq, (unsigned long long)walked_h[si],
+                    (unsigned long long)plan[si].s.n_records);
     } else if (hs.limit) {
       status = (hs.limit & 2) ? fail(OWL_ERR_CAPACITY, "a traced warp visits more than %d distinct basic blocks",
                                      owl_fold_max_bbs())
@@ -861,15 +877,13 @@ OWL_API owl_status owl_filter_inputs(owl_ctx* ctx, const uint32_t* runs, size_t 
   return OWL_OK;
 }
 
-OWL_API owl_status owl_leak_test(owl_ctx* ctx, const owl_adcfg* f, const owl_adcfg* r, double significance,
-                                 owl_leak** leaks, size_t* n_leaks) {
-  if (!ctx || !f || !r || !leaks || !n_leaks) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
-  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+namespace {
+
+/* kernel leaks: unaligned invocations, or aligned with different counts (reading R12), in alignment
+   order */
+void kernel_leaks(const owl_adcfg* f, const owl_adcfg* r, const Alignment& al, std::vector<owl_leak>& out) {
   const uint32_t NA = 0xFFFFFFFFu;
   const double nan = std::nan("");
-  Alignment al = align(f, r);
-  std::vector<owl_leak> out;
-  /* kernel leaks: unaligned invocations, or aligned with different counts (reading R12) */
   for (const OwlEdit& o : al.ops) {
     owl_leak l;
     memset(&l, 0, sizeof l);
@@ -895,6 +909,37 @@ OWL_API owl_status owl_leak_test(owl_ctx* ctx, const owl_adcfg* f, const owl_adc
       }
     }
   }
+}
+
+/* CF rows, then DF rows, each by (alignment position of the fix slot, bb, ins); a DF location keeps its
+   min-p row, ties -> smallest j (reading R14).  `rows` may hold several rows of one DF location (owners of
+   the multi-GPU path split its visits j); CF rows are unique per (slot, bb). */
+void order_ks_leaks(const Alignment& al, std::vector<owl_leak>& rows, std::vector<owl_leak>& out) {
+  auto pos = [&](const owl_leak& l) { return l.slot_fix < al.pos_of_f.size() ? al.pos_of_f[l.slot_fix] : -1; };
+  std::vector<owl_leak> cf, df;
+  for (const owl_leak& l : rows) (l.kind == OWL_LEAK_CONTROL_FLOW ? cf : df).push_back(l);
+  std::stable_sort(cf.begin(), cf.end(), [&](const owl_leak& a, const owl_leak& b) {
+    return std::make_tuple(pos(a), a.bb) < std::make_tuple(pos(b), b.bb);
+  });
+  std::stable_sort(df.begin(), df.end(), [&](const owl_leak& a, const owl_leak& b) {
+    return std::make_tuple(pos(a), a.bb, a.ins, a.p, a.j) < std::make_tuple(pos(b), b.bb, b.ins, b.p, b.j);
+  });
+  out.insert(out.end(), cf.begin(), cf.end());
+  for (size_t i = 0; i < df.size(); ++i) /* first of each location = min p, then smallest j */
+    if (i == 0 || pos(df[i]) != pos(df[i - 1]) || df[i].bb != df[i - 1].bb || df[i].ins != df[i - 1].ins)
+      out.push_back(df[i]);
+}
+
+}  // namespace
+
+OWL_API owl_status owl_leak_test(owl_ctx* ctx, const owl_adcfg* f, const owl_adcfg* r, double significance,
+                                 owl_leak** leaks, size_t* n_leaks) {
+  if (!ctx || !f || !r || !leaks || !n_leaks) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
+  const uint32_t NA = 0xFFFFFFFFu;
+  Alignment al = align(f, r);
+  std::vector<owl_leak> out;
+  kernel_leaks(f, r, al, out);
   std::vector<owl_ks_row> rows;
   std::vector<int> pos;
   owl_status s = run_ks(ctx, f, r, significance, al, rows, pos);
@@ -908,25 +953,73 @@ OWL_API owl_status owl_leak_test(owl_ctx* ctx, const owl_adcfg* f, const owl_adc
     l.n = k.n; l.m = k.m; l.K_lo = k.K_lo; l.K_hi = k.K_hi; l.D = k.D; l.p = k.p;
     return l;
   };
-  /* CF leaks at the node's BB */
+  /* CF leaks at the node's BB; DF leak at (slot, bb, ins) if any visit j fails, representative =
+     min p, ties -> smallest j (R14) */
+  std::vector<owl_leak> failing;
   for (const owl_ks_row& k : rows)
-    if (k.fail && k.kind == OWL_LEAK_CONTROL_FLOW) out.push_back(to_leak(k, OWL_LEAK_CONTROL_FLOW));
-  /* DF leak at (slot, bb, ins) if any visit j fails; representative = min p, ties -> smallest j (R14) */
-  size_t i = 0;
-  while (i < rows.size()) {
-    if (rows[i].kind != OWL_LEAK_DATA_FLOW) { ++i; continue; }
-    size_t e = i;
-    int best = -1;
-    while (e < rows.size() && rows[e].kind == OWL_LEAK_DATA_FLOW && pos[e] == pos[i] && rows[e].bb == rows[i].bb &&
-           rows[e].ins == rows[i].ins) {
-      if (rows[e].fail && (best < 0 || rows[e].p < rows[best].p)) best = (int)e;
-      ++e;
-    }
-    if (best >= 0) out.push_back(to_leak(rows[best], OWL_LEAK_DATA_FLOW));
-    i = e;
-  }
+    if (k.fail) failing.push_back(to_leak(k, k.kind));
+  order_ks_leaks(al, failing, out);
   *leaks = host_copy(out);
   *n_leaks = out.size();
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_merge_leaks(owl_ctx* ctx, const owl_adcfg* f, const owl_adcfg* r, const owl_leak* parts,
+                                   size_t n_parts, owl_leak** leaks, size_t* n_leaks) {
+  if (!ctx || !f || !r || !leaks || !n_leaks || (n_parts && !parts)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  Alignment al = align(f, r);
+  std::vector<owl_leak> out, ks;
+  kernel_leaks(f, r, al, out); /* replicated on every owner: recomputed here from the slot tables */
+  for (size_t i = 0; i < n_parts; ++i) {
+    const owl_leak& l = parts[i];
+    if (l.kind == OWL_LEAK_KERNEL) continue;
+    if (l.kind > OWL_LEAK_DATA_FLOW || l.slot_fix >= al.pos_of_f.size() || al.pos_of_f[l.slot_fix] < 0)
+      return fail(OWL_ERR_INVALID_ARG, "leak row %zu: kind %u / fix slot %u not an aligned slot of e_fix", i, l.kind,
+                  l.slot_fix);
+    ks.push_back(l);
+  }
+  order_ks_leaks(al, ks, out);
+  *leaks = host_copy(out);
+  *n_leaks = out.size();
+  return OWL_OK;
+}
+
+OWL_API owl_status owl_merge_diffs(owl_ctx* ctx, const owl_adcfg* a, const owl_adcfg* b, const owl_diff* parts,
+                                   size_t n_parts, owl_diff** rows, size_t* n_rows) {
+  if (!ctx || !a || !b || !rows || !n_rows || (n_parts && !parts)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
+  std::vector<owl_diff> out;
+  for (size_t i = 0; i < n_parts; ++i) {
+    if (parts[i].table > OWL_TABLE_SLOT) return fail(OWL_ERR_INVALID_ARG, "diff row %zu: table %u", i, parts[i].table);
+    if (parts[i].table != OWL_TABLE_SLOT) out.push_back(parts[i]);
+  }
+  /* canonical (table, key) order: the owners' rows are disjoint (each cell lives on one owner) */
+  auto key = [](const owl_diff& d) {
+    return d.table == OWL_TABLE_NODE   ? std::make_tuple(d.table, d.slot, d.bb, 0u, 0u, 0u, 0u, (uint64_t)0)
+           : d.table == OWL_TABLE_EDGE ? std::make_tuple(d.table, d.slot, d.prev, d.next, 0u, 0u, 0u, (uint64_t)0)
+           : d.table == OWL_TABLE_TRIPLE ? std::make_tuple(d.table, d.slot, d.bb, d.prev, d.next, 0u, 0u, (uint64_t)0)
+                                         : std::make_tuple(d.table, d.slot, d.bb, d.ins, d.j, 0u, 0u, d.x);
+  };
+  std::sort(out.begin(), out.end(), [&](const owl_diff& x, const owl_diff& y) { return key(x) < key(y); });
+  /* slot rows (replicated): recomputed from the slot tables, exactly as owl_diff_adcfg writes them */
+  {
+    std::map<std::pair<uint32_t, uint64_t>, std::pair<uint64_t, uint64_t>> all;
+    for (uint32_t sl : a->slots.order) all[{sl, a->slots.kid[sl]}].first = a->slots.count[sl];
+    for (uint32_t sl : b->slots.order) all[{sl, b->slots.kid[sl]}].second = b->slots.count[sl];
+    for (auto& e : all)
+      if (e.second.first != e.second.second) {
+        owl_diff r;
+        memset(&r, 0, sizeof r);
+        r.table = OWL_TABLE_SLOT;
+        r.slot = e.first.first;
+        r.bb = r.ins = r.j = r.prev = r.next = 0xFFFFFFFFu;
+        r.x = e.first.second;
+        r.count_a = e.second.first;
+        r.count_b = e.second.second;
+        out.push_back(r);
+      }
+  }
+  *rows = host_copy(out);
+  *n_rows = out.size();
   return OWL_OK;
 }
 

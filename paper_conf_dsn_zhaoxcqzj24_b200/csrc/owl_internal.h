@@ -75,6 +75,9 @@ struct FoldSeg {
   uint32_t slot;      /* evidence slot of this invocation */
   uint32_t n_warps;
   uint32_t* seen;     /* bitmap of n_warps bits (warp-major check), zeroed */
+  unsigned long long* walked; /* records the fold walked in this segment, zeroed; = n iff every record was
+                                 walked exactly once (with `seen`: the warp-major check) */
+  const unsigned long long* perm; /* channel-order segment bucketed by warp: caller's index of each record */
   uint32_t seg_index; /* position in the build's (run, seq)-sorted segment list */
   uint32_t _pad;
 };

@@ -13,8 +13,8 @@ The path shards by run (runs are independent up to integer sums) and has one exc
 4. ``owner_evidence``: ``owl_partition_evidence`` packs every cell by owner(attr) = mix64(attr) mod world,
    ``all_to_all_single`` moves the counts and then the cells, ``owl_absorb_evidence`` sums what arrived:
    each KS attribute now lives whole on one rank (integer sums: bit-identical to one GPU).
-5. ``leak_test`` / ``diff``: each owner tests / diffs its attributes; rows are gathered and put back in
-   canonical order.  The kernel test and the slot rows are replicated on every rank; rank 0 keeps them.
+5. ``leak_test`` / ``diff``: each owner tests / diffs its attributes; rows are all-gathered and merged by the
+   library (``owl_merge_leaks`` / ``owl_merge_diffs``) into exactly the one-GPU result.
 
 Only argument marshalling happens here: every step on the data runs in libowl's kernels.
 """
@@ -92,38 +92,17 @@ def gather_rows(rows: np.ndarray, group=None) -> np.ndarray:
     return np.concatenate(parts) if parts else rows[:0].copy()
 
 
-def merge_leaks(parts: list) -> np.ndarray:
-    """Owners' leak rows (rank 0's first) -> one list: kernel rows once (replicated), then CF, DF rows by
-    (slot, bb, ins).  Owners split a DF location's visits j (attribute = (slot, bb, ins, j)), so each may
-    report the location: keep the row of the minimum p, ties -> smallest j (reading R14), as one GPU does."""
-    kernel = parts[0][parts[0]["kind"] == 0]  # replicated, already in the library's (alignment) order
-    allr = np.concatenate([p[p["kind"] != 0] for p in parts])
-    allr = allr[np.lexsort((allr["j"], allr["p"], allr["ins"], allr["bb"], allr["slot_rnd"], allr["slot_fix"],
-                            allr["kind"]))]
-    if len(allr):
-        k = np.stack([allr["kind"], allr["slot_fix"], allr["slot_rnd"], allr["bb"], allr["ins"]], axis=1)
-        first = np.ones(len(allr), dtype=bool)
-        first[1:] = np.any(k[1:] != k[:-1], axis=1) | (allr["kind"][1:] != 2)
-        allr = allr[first]
-    # CF / DF rows by (kind, slot, bb, ins): the one-GPU order whenever slot ids follow the alignment
-    return np.concatenate([kernel, allr[np.lexsort((allr["ins"], allr["bb"], allr["slot_fix"], allr["kind"]))]])
-
-
-def merge_diffs(parts: list) -> np.ndarray:
-    """Owners' diff rows -> canonical (table, key) order; slot rows (table 4) are replicated: rank 0's."""
-    keep = [parts[0]] + [p[p["table"] != 4] for p in parts[1:]]
-    allr = np.concatenate(keep)
-    return allr[np.lexsort((allr["x"], allr["next"], allr["prev"], allr["j"], allr["ins"], allr["bb"], allr["slot"],
-                            allr["table"]))]
-
-
 def leak_test(ctx, owned_f, owned_r, significance: float, group=None) -> np.ndarray:
+    """Each owner tests its attributes; the rows are all-gathered and merged by the library
+    (owl_merge_leaks: kernel rows from the replicated slot tables, CF / DF rows by alignment position, a DF
+    location split across owners keeps its min-p visit, ties -> smallest j)."""
     parts = [None] * dist.get_world_size(group)
     dist.all_gather_object(parts, ctx.leak_test(owned_f, owned_r, significance), group=group)
-    return merge_leaks(parts)
+    return ctx.merge_leaks(owned_f, owned_r, parts)
 
 
 def diff(ctx, owned_a, owned_b, group=None) -> np.ndarray:
+    """Each owner diffs its cells; rows all-gathered, merged into canonical order by owl_merge_diffs."""
     parts = [None] * dist.get_world_size(group)
     dist.all_gather_object(parts, ctx.diff(owned_a, owned_b), group=group)
-    return merge_diffs(parts)
+    return ctx.merge_diffs(owned_a, owned_b, parts)

@@ -142,3 +142,69 @@ def interleave_random(rng, rec):
         if not queues[k]:
             queues.pop(k)
     return rec[np.array(order)]
+
+
+# ---- hand-worked leak-test cases (tests/golden/leak_localization.json) ------------------------------
+NA = 0xFFFFFFFF
+
+
+def dsl_records(visits, n_warps):
+    """Warp-major records of one invocation: every warp runs `visits` = [[bb, [[ins, lanes, base], ...]], ...];
+    lane l < lanes of instruction ins accesses x = (3 << 60) | (base + 4 l)."""
+    rows = []
+    for w in range(n_warps):
+        for bb, mems in visits:
+            rows.append(bb_rec(w, bb))
+            for ins, lanes, base in mems:
+                for lane in range(lanes):
+                    rows.append(mem_rec(w, bb, ins, lane, (3 << 60) | (base + 4 * lane)))
+    return to_records(rows)
+
+
+def golden_case_invocations(case):
+    """[(run, class, seq, n_warps, kernel_id, records)] of a leak_localization.json case."""
+    out = []
+    for run, cls, names in case["runs"]:
+        for seq, name in enumerate(names):
+            nw = case["n_warps"][name]
+            out.append((run, cls, seq, nw, case["kernels"][name], dsl_records(case["bodies"][name][str(cls)], nw)))
+    return out
+
+
+def golden_expected_rows(case):
+    """Expected leak rows with NA / nan / closed-form p resolved: list of dicts."""
+    import math
+    rows = []
+    for e in case["expected"]:
+        r = {}
+        for k, v in e.items():
+            if k == "kernel":
+                r["kernel_id"] = case["kernels"][v]
+            elif v == "NA":
+                r[k] = NA
+            elif v == "nan":
+                r[k] = float("nan")
+            elif k == "p" and isinstance(v, str):
+                assert v.startswith("2*exp(-") and v.endswith(")"), v
+                r[k] = 2.0 * math.exp(-float(v[7:-1]))
+            else:
+                r[k] = v
+        rows.append(r)
+    return rows
+
+
+def assert_leaks_equal_golden(got, case):
+    """Every field of every leak row against the hand-worked expectation (p: closed form, 1e-12 relative)."""
+    import math
+    want = golden_expected_rows(case)
+    assert len(got) == len(want), (len(got), len(want))
+    for g, w in zip(got, want):
+        for f in ("kind", "slot_fix", "slot_rnd", "bb", "ins", "j", "kernel_id", "n", "m"):
+            assert int(g[f]) == int(w[f]), (f, int(g[f]), w)
+        K = int(g["K_lo"]) | (int(g["K_hi"]) << 64)
+        assert K == int(w["K"]), (K, w)
+        for f in ("D", "p"):
+            if math.isnan(w[f]):
+                assert math.isnan(float(g[f])), (f, g[f], w)
+            else:
+                assert abs(float(g[f]) - w[f]) <= 1e-12 * abs(w[f]), (f, float(g[f]), w)

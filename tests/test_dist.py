@@ -1,13 +1,12 @@
 """Multi-GPU host logic (paper_conf_dsn_zhaoxcqzj24_b200/dist.py) with world-size-2 gloo on CPU: run sharding,
-kernel-sequence gathering, the byte all-to-all of the exchange, and the canonical merge of owners' rows."""
+kernel-sequence gathering and the byte all-to-all of the exchange.  (The merge of the owners' rows is a
+library call, owl_merge_leaks / owl_merge_diffs, checked against the oracle in tests/test_gpu_sequences.py.)"""
 import os
 import socket
 
-import numpy as np
 import pytest
 import torch.multiprocessing as mp
 
-from oracle import oracle
 
 
 def _free_port():
@@ -69,23 +68,3 @@ def test_shard_balanced_and_contiguous():
             parts = [D.shard(range(n), world, r) for r in range(world)]
             assert sum(parts, []) == list(range(n))
             assert max(map(len, parts)) - min(map(len, parts)) <= 1
-
-
-def test_merge_rows_canonical_order():
-    """Owners' rows -> one canonical list: replicated kernel / slot rows kept once (rank 0's)."""
-    from paper_conf_dsn_zhaoxcqzj24_b200 import dist as D
-    L = np.zeros(5, dtype=oracle.LEAK_DTYPE)
-    L["kind"] = [0, 2, 1, 2, 2]
-    L["slot_fix"] = [0, 0, 0, 0, 1]
-    L["bb"] = [9, 3, 1, 1, 0]
-    L["ins"] = [9, 2, 0, 5, 0]
-    r0, r1 = L[[0, 1, 4]], L[[0, 2, 3]]  # kernel row replicated
-    m = D.merge_leaks([r0, r1])
-    assert list(m["kind"]) == [0, 1, 2, 2, 2] and list(m["bb"]) == [9, 1, 1, 3, 0]
-    Dr = np.zeros(4, dtype=oracle.DIFF_DTYPE)
-    Dr["table"] = [3, 0, 4, 3]
-    Dr["slot"] = [0, 0, 0, 0]
-    Dr["bb"] = [2, 1, 0xFFFFFFFF, 1]
-    Dr["x"] = [5, 0, 7, 9]
-    m = D.merge_diffs([Dr[[0, 2]], Dr[[1, 2, 3]]])
-    assert list(m["table"]) == [0, 3, 3, 4] and list(m["bb"][1:3]) == [1, 2]

@@ -4,8 +4,6 @@ Bar (BASELINE.json north_star): canonical A-DCFG dumps (node / ed
 slot table) and diff rows bit-exact; KS K exact and D bit-identical; p within 1e-9 relative (x when p underflows);
 leak verdicts and locations identical except where p is within 1e-9 of the threshold.
 """
-import math
-
 import numpy as np
 import pytest
 
@@ -20,8 +18,8 @@ if not torch.cuda.is_available():  # pragma: no cover
     pytest.skip("needs a CUDA device", allow_module_level=True)
 
 from paper_conf_dsn_zhaoxcqzj24_b200 import api  # noqa: E402
-
-SIG = 0.05
+from tests.gpu_common import (SIG, _build_and_compare, _gpu_segments, _oracle_segments, _runs_of,  # noqa: E402
+                              assert_ks_parity, assert_leak_parity)
 
 
 @pytest.fixture(scope="module")
@@ -29,94 +27,9 @@ def ctx():
     return api.Context(0)
 
 
-def _gpu_segments(p, runs, interleaved=False):
-    segs = []
-    for r in runs:
-        for m in tracegen.run_segments(p, r):
-            if interleaved:
-                rec = tracegen.interleave(tracegen.host_records(p, r, m.seq))
-                buf = torch.from_numpy(rec.view(np.uint8).copy()).cuda()
-                segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, len(rec), flags=0))
-            else:
-                buf, n = tracegen.device_records(p, r, m.seq)
-                segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, n))
-    return segs
-
-
-def _oracle_segments(p, runs):
-    out = {0: [], 1: []}
-    for r in runs:
-        for m in tracegen.run_segments(p, r):
-            out[m.input_class].append(oracle.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id,
-                                                     tracegen.host_records(p, r, m.seq)))
-    return out
-
-
-def _runs_of(p, cls):
-    return [r for r in range(p.n_runs) if tracegen.run_class(p, r) == cls]
-
-
-def _same_p(a, b):
-    if a == b:
-        return True
-    if a < 2.2250738585072014e-308 or b < 2.2250738585072014e-308:
-        xa, xb = -math.log(max(a, 5e-324) / 2), -math.log(max(b, 5e-324) / 2)
-        return abs(xa - xb) <= 1e-9 * max(abs(xa), abs(xb)) or (a == 0 and b == 0)
-    return abs(a - b) <= 1e-9 * max(abs(a), abs(b))
-
-
-def assert_ks_parity(g, o):
-    assert len(g) == len(o)
-    for f in ("kind", "slot_fix", "slot_rnd", "bb", "ins", "j", "n", "m", "K_lo", "K_hi"):
-        assert np.array_equal(g[f], o[f]), f
-    assert np.array_equal(g["D"].view(np.uint64), o["D"].view(np.uint64)), "D must be bit-identical"
-    for i in range(len(g)):
-        assert _same_p(float(g["p"][i]), float(o["p"][i])), (i, g["p"][i], o["p"][i])
-        if g["fail"][i] != o["fail"][i]:
-            assert abs(float(o["p"][i]) - SIG) <= 1e-9 * SIG, i
-
-
-def assert_leak_parity(g, o):
-    near = [i for i in range(len(o)) if o["kind"][i] != 0 and abs(float(o["p"][i]) - SIG) <= 1e-9 * SIG]
-    assert not near, "a p-value inside the tolerance band of the threshold: compare verdicts by hand"
-    assert len(g) == len(o)
-    for f in ("kind", "slot_fix", "slot_rnd", "bb", "ins", "j", "kernel_id", "n", "m", "K_lo", "K_hi"):
-        assert np.array_equal(g[f], o[f]), f
-    ks = g["kind"] != 0
-    assert np.array_equal(g["D"][ks].view(np.uint64), o["D"][ks].view(np.uint64))
-    for i in np.flatnonzero(ks):
-        assert _same_p(float(g["p"][i]), float(o["p"][i]))
-
-
-def _build_and_compare(ctx, p, runs=None, interleaved=False):
-    runs = list(range(p.n_runs)) if runs is None else runs
-    segs = _gpu_segments(p, runs, interleaved)
-    ctx.ingest(segs)
-    try:
-        rf = [r for r in runs if tracegen.run_class(p, r) == 0]
-        rr = [r for r in runs if tracegen.run_class(p, r) == 1]
-        ef, er = ctx.build(rf), ctx.build(rr)
-        osg = _oracle_segments(p, runs)
-        of, orr = oracle.build(osg[0]), oracle.build(osg[1])
-        bf, bo = ef.export(), of.export()
-        if bf != bo:
-            pf, po = H.parse_blob(bf), H.parse_blob(bo)
-            for t in ("slots", "node", "edge", "triple", "addr"):
-                assert len(pf[t]) == len(po[t]) and np.array_equal(pf[t], po[t]), t
-        assert bf == bo
-        assert er.export() == orr.export()
-        assert_ks_parity(ctx.ks_tests(ef, er, SIG), oracle.ks_tests(of, orr, SIG))
-        assert_leak_parity(ctx.leak_test(ef, er, SIG), oracle.leak_test(of, orr, SIG))
-        gd, od = ctx.diff(ef, er), oracle.diff(of, orr)
-        assert len(gd) == len(od) and np.array_equal(gd, od)
-        return ef, er, of, orr
-    finally:
-        ctx.forget_runs(runs)
-
-
 def test_generator_device_equals_host():
     """T3: the counter-based generator gives byte-identical records on host and device."""
-    for cfg, div in ((1, 1), (2, 64), (3, 16), (4, 128), (5, 32)):
+    for cfg, div in ((1, 1), (2, 64), (3, 16), (4, 128), (5, 32), (9, 16)):
         p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=1, runs_rnd=1)
         for r in (0, 1):
             for m in tracegen.run_segments(p, r):
@@ -383,7 +296,7 @@ def test_rq2_workloads_parity(ctx, cfg, threads):
     _build_and_compare(ctx, p)
 
 
-@pytest.mark.parametrize("cfg,div,nf,nr", [(2, 64, 3, 3), (4, 256, 2, 3)])
+@pytest.mark.parametrize("cfg,div,nf,nr", [(2, 64, 3, 3), (4, 256, 2, 3), (9, 8, 3, 5)])
 def test_sharded_exchange_equals_one_gpu(cfg, div, nf, nr):
     """§8(e) on one GPU: two 'ranks' (two contexts) each fold a shard of the runs with agreed slots, partition
     their partial evidences by owner, the buckets are exchanged (the all-to-all, done by hand), and each owner
@@ -423,8 +336,10 @@ def test_sharded_exchange_equals_one_gpu(cfg, div, nf, nr):
             keep.append(recv)
             owned[(owner, cls)] = ctxs[owner].absorb(parts[(owner, cls)], recv.data_ptr() if recv.numel() else None,
                                                      rb, owner)
-    leaks = D.merge_leaks([ctxs[o].leak_test(owned[(o, 0)], owned[(o, 1)], SIG) for o in range(world)])
-    diffs = D.merge_diffs([ctxs[o].diff(owned[(o, 0)], owned[(o, 1)]) for o in range(world)])
+    leaks = ctxs[0].merge_leaks(owned[(0, 0)], owned[(0, 1)],
+                                [ctxs[o].leak_test(owned[(o, 0)], owned[(o, 1)], SIG) for o in range(world)])
+    diffs = ctxs[0].merge_diffs(owned[(0, 0)], owned[(0, 1)],
+                                [ctxs[o].diff(owned[(o, 0)], owned[(o, 1)]) for o in range(world)])
     ks = np.concatenate([ctxs[o].ks_tests(owned[(o, 0)], owned[(o, 1)], SIG) for o in range(world)])
     osg = _oracle_segments(p, runs)
     of, orr = oracle.build(osg[0]), oracle.build(osg[1])
@@ -519,3 +434,100 @@ def test_hcf_reading_invalid(ctx):
     with pytest.raises(api.OwlError, match="OWL_ERR_INVALID_ARG"):
         ctx.set_config(hcf_reading=2)
     ctx.set_config()
+
+
+_MISFLAG_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, {root!r})
+import tracegen
+from tests import helpers as H
+from paper_conf_dsn_zhaoxcqzj24_b200 import api
+p = tracegen.Params.preset(2, grid_div=16, runs_fix=1, runs_rnd=0)
+rec = tracegen.host_records(p, 0, 0)
+variants = {{"interleaved": tracegen.interleave(rec)}}
+g = rec["gwarp"]
+b1, b2, b3 = (int(np.flatnonzero(g == w)[0]) for w in (1, 2, 3))
+mid = (b1 + b2) // 2  # warp 2's block moved into the middle of warp 1's (warp 1 then starts twice)
+variants["split_warp"] = np.concatenate([rec[:mid], rec[b2:b3], rec[mid:b2], rec[b3:]])
+# 100 records of the last warp hidden 50 records past a fold-tile boundary (2^15) inside another warp's block:
+# closer than the tile search's sample spacing, so only the walked-record count can notice them
+last = int(np.flatnonzero(g == g.max())[0])
+t = 1 << 15
+variants["hidden_block"] = np.concatenate([rec[:t + 50], rec[last:last + 100], rec[t + 50:last], rec[last + 100:]])
+assert g[t - 1] == g[t + 60]
+ctx = api.Context(0)
+for name, r in variants.items():
+    buf = torch.from_numpy(r.view(np.uint8).copy()).cuda()
+    ctx.ingest([api.Segment(0, 0, 0, 128, 10, buf, len(r), flags=api.OWL_SEG_WARP_MAJOR)])
+    try:
+        ctx.build([0])
+        print(name, "BUILT")
+    except api.OwlError as e:
+        print(name, str(e).split(":")[0])
+    finally:
+        ctx.forget_runs([0])
+"""
+
+
+def test_warp_major_misflag_detected():
+    """Segments wrongly flagged OWL_SEG_WARP_MAJOR (> 2^15 records, several fold tiles) fail with
+    OWL_ERR_INVALID_ARG: channel order, one warp's block moved inside another's, and a short block hidden just
+    past a tile boundary.  No hang (the run is a subprocess under a timeout), no silently skipped record."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _MISFLAG_SCRIPT.format(root=root)], capture_output=True, text=True,
+                       timeout=300, cwd=root)
+    assert r.returncode == 0, r.stderr
+    lines = dict(ln.split(" ", 1) for ln in r.stdout.strip().splitlines())
+    assert lines == {"interleaved": "OWL_ERR_INVALID_ARG", "split_warp": "OWL_ERR_INVALID_ARG",
+                     "hidden_block": "OWL_ERR_INVALID_ARG"}, r.stdout
+
+
+def test_channel_order_first_bad_record(ctx):
+    """Channel order with two malformed records: the report names the first in the caller's order (as the oracle
+    does), although bucketing by warp puts the other one first."""
+    rec = tracegen.interleave(H.w1_records(), burst=2)
+    w0 = [i for i in range(len(rec)) if rec["gwarp"][i] == 0 and rec["meta"][i] >> 31]
+    w1 = [i for i in range(len(rec)) if rec["gwarp"][i] == 1 and rec["meta"][i] >> 31]
+    late0, early1 = w0[-1], w1[0]
+    assert early1 < late0
+    for i in (late0, early1):
+        rec["addr"][i] = np.uint64(12) << np.uint64(60)
+    with pytest.raises(oracle.OracleError) as eo:
+        oracle.build([oracle.Segment(0, 0, 0, 2, 10, rec)])
+    assert f"record {early1}:" in str(eo.value)
+    buf = torch.from_numpy(rec.view(np.uint8).copy()).cuda()
+    ctx.ingest([api.Segment(0, 0, 0, 2, 10, buf, len(rec), flags=0)])
+    try:
+        with pytest.raises(api.OwlError, match="OWL_ERR_MALFORMED_TRACE") as eg:
+            ctx.build([0])
+        assert str(eo.value).split(": ", 1)[1] in str(eg.value)
+    finally:
+        ctx.forget_runs([0])
+
+
+@pytest.mark.parametrize("cfg,div,interleaved", [(2, 32, False), (5, 32, True), (4, 256, False)])
+def test_host_records_e2e_path(ctx, cfg, div, interleaved):
+    """OWL_SEG_HOST_RECORDS (the bench's e2e leg): host buffers staged by the library give the oracle's result."""
+    p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=2, runs_rnd=2)
+    runs = list(range(p.n_runs))
+    segs = []
+    for r in runs:
+        for m in tracegen.run_segments(p, r):
+            rec = tracegen.host_records(p, r, m.seq)
+            if interleaved:
+                rec = tracegen.interleave(rec)
+            host = torch.from_numpy(rec.view(np.uint8).copy()).pin_memory()
+            flags = api.OWL_SEG_HOST_RECORDS | (0 if interleaved else api.OWL_SEG_WARP_MAJOR)
+            segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, host, len(rec), flags=flags))
+    ctx.ingest(segs)
+    try:
+        ef, er = ctx.build(_runs_of(p, 0)), ctx.build(_runs_of(p, 1))
+        osg = _oracle_segments(p, runs)
+        of, orr = oracle.build(osg[0]), oracle.build(osg[1])
+        assert ef.export() == of.export() and er.export() == orr.export()
+        assert_leak_parity(ctx.leak_test(ef, er, SIG), oracle.leak_test(of, orr, SIG))
+    finally:
+        ctx.forget_runs(runs)

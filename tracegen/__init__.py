@@ -30,9 +30,11 @@ CONFIGS = {
     6: dict(runs_fix=1, runs_rnd=0, grid_div=1, threads=1024),  # pattern 2: dummy S-box program
     7: dict(runs_fix=1, runs_rnd=0, grid_div=1, threads=1024),  # pattern 3: thread-distinct pixels
     8: dict(runs_fix=1, runs_rnd=0, grid_div=1, threads=1024),  # pattern 1: fixed threads
+    # kernel-sequence model (Myers on repeated kernel ids, mid-sequence insertions / deletions)
+    9: dict(runs_fix=8, runs_rnd=8, grid_div=1),
 }
 CONFIG_NAMES = {1: "C1-toy", 2: "C2-aes128-ttable", 3: "C3-rsa-modexp", 4: "C4-pytorch-ops", 5: "C5-nvjpeg-decode",
-                6: "RQ2-sbox", 7: "RQ2-pixel", 8: "RQ2-fixed-threads"}
+                6: "RQ2-sbox", 7: "RQ2-pixel", 8: "RQ2-fixed-threads", 9: "C9-kernel-sequence-model"}
 
 
 class _Params(ctypes.Structure):

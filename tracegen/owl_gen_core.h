@@ -23,6 +23,8 @@
  *                     (launched only if the input is not all-zero: RND all-zero with probability 1/2)
  *   C5 nvJPEG-shaped  Huffman decode (8,192 thr, image-dependent symbol counts and LUT lookups) + IDCT
  *                     (128,000 thr)
+ *   9  kernel-sequence model: a secret-dependent launch sequence over the C4 kernel bodies with a
+ *                     repeated kernel (3-4x) and mid-sequence insertions / a trailing deletion (Myers)
  * Runs: run r is FIX or RND interleaved (r even FIX / odd RND while both classes have runs left);
  * FIX reuses one secret for all its runs, RND draws a fresh secret per run.  Non-secret
  * inputs (plaintexts, images' geometry, conv inputs) are fixed per thread across runs.
@@ -45,7 +47,7 @@ typedef struct {
 } og_record;
 
 typedef struct {
-  uint32_t config;   /* 1..5 (BASELINE configs), 6..8 (RQ2 sweep) */
+  uint32_t config;   /* 1..5 (BASELINE configs), 6..8 (RQ2 sweep), 9 (kernel-sequence model) */
   uint32_t grid_div; /* every kernel's block count is divided by this (min 1 block); 1 = paper shape */
   uint32_t runs_fix;
   uint32_t runs_rnd;
@@ -60,7 +62,7 @@ enum { OG_T_NONE = 0, OG_T_LOCAL = 1, OG_T_GENERIC = 2, OG_T_GLOBAL = 3, OG_T_SH
 
 /* stream tags of the counter-based generator */
 enum { OG_TAG_FIX = 1, OG_TAG_RND, OG_TAG_PT, OG_TAG_NOISE, OG_TAG_STATE, OG_TAG_EXP, OG_TAG_TOK, OG_TAG_ZERO,
-       OG_TAG_NS, OG_TAG_CODE, OG_TAG_KID, OG_TAG_PERM };
+       OG_TAG_NS, OG_TAG_CODE, OG_TAG_KID, OG_TAG_PERM, OG_TAG_SEQ };
 
 OG_HD uint64_t og_mix(uint64_t x) {
   x += 0x9E3779B97F4A7C15ull;
@@ -99,18 +101,38 @@ enum { OG_K_TOY = 0, OG_K_AES, OG_K_RSA, OG_K_EMBED, OG_K_CONV, OG_K_SOFTMAX, OG
        OG_K_SBOX, OG_K_PIXEL, OG_K_REPR };
 
 OG_HD int og_c4_allzero(const og_params* p, uint32_t r) {
-  return og_run_class(p, r) == OG_RND && (og_h2(og_run_secret(p, r), OG_TAG_ZERO) & 1u);
+  return p->config == 4 && og_run_class(p, r) == OG_RND && (og_h2(og_run_secret(p, r), OG_TAG_ZERO) & 1u);
+}
+/* config 9 (kernel-sequence model): the host code of a small model launches a secret-dependent kernel
+   sequence E L [G] L [G] L [L] [N] — the layer kernel L repeats 3-4 times, the gate kernel G is inserted
+   mid-sequence 0-2 times, the final N is skipped on one secret bit — so the Myers alignment of runs
+    sees repeated kernel ids and mid-sequence insertions / deletions.  Returns the length. */
+OG_HD uint32_t og_c9_seq(const og_params* p, uint32_t r, uint32_t* ks) {
+  const uint64_t b = og_h2(og_run_secret(p, r), OG_TAG_SEQ);
+  uint32_t n = 0;
+  ks[n++] = OG_K_EMBED;
+  ks[n++] = OG_K_SOFTMAX;
+  if (b & 1u) ks[n++] = OG_K_NONZERO;
+  ks[n++] = OG_K_SOFTMAX;
+  if (b & 2u) ks[n++] = OG_K_NONZERO;
+  ks[n++] = OG_K_SOFTMAX;
+  if (b & 4u) ks[n++] = OG_K_SOFTMAX;
+  if (!(b & 8u)) ks[n++] = OG_K_CONV;
+  return n;
 }
 OG_HD uint32_t og_n_seq(const og_params* p, uint32_t r) {
+  uint32_t ks[8];
   switch (p->config) {
     case 4: return og_c4_allzero(p, r) ? 3u : 4u;
     case 5: return 2u;
+    case 9: return og_c9_seq(p, r, ks);
     default: return 1u;
   }
 }
 OG_HD uint32_t og_seq_kernel(const og_params* p, uint32_t r, uint32_t seq) {
-  (void)r;
+  uint32_t ks[8];
   switch (p->config) {
+    case 9: return og_c9_seq(p, r, ks) > seq ? ks[seq] : OG_K_CONV;
     case 1: return OG_K_TOY;
     case 2: return OG_K_AES;
     case 3: return OG_K_RSA;
@@ -125,6 +147,7 @@ OG_HD uint32_t og_seq_kernel(const og_params* p, uint32_t r, uint32_t seq) {
 OG_HD uint64_t og_kernel_id(const og_params* p, uint32_t k) { return og_h3(0x0DC0FFEEull, OG_TAG_KID, p->config * 16u + k); }
 OG_HD uint32_t og_kernel_wpb(uint32_t k) { return k == OG_K_TOY ? 4u : 8u; }
 OG_HD uint32_t og_kernel_blocks(const og_params* p, uint32_t k) {
+  if (p->config == 9) return og_blocks(p, 16); /* 128 warps per kernel */
   switch (k) {
     case OG_K_TOY: return og_blocks(p, 2);
     case OG_K_AES: return og_blocks(p, 256);
@@ -459,7 +482,7 @@ OG_HD uint64_t og_warp(const og_params* p, uint32_t r, uint32_t seq, uint32_t gw
     case 1: og_warp_c1(p, r, &e); break;
     case 2: og_warp_c2(p, r, &e); break;
     case 3: og_warp_c3(p, r, &e); break;
-    case 4: og_warp_c4(p, r, k, &e); break;
+    case 4: case 9: og_warp_c4(p, r, k, &e); break;
     case 6: case 7: case 8: og_warp_rq2(p, r, k, &e); break;
     default: og_warp_c5(p, r, k, &e); break;
   }
