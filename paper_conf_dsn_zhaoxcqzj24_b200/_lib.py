@@ -66,7 +66,10 @@ def load():
             raise ImportError(f"libowl.so not found at {LIB_PATH}: run `python __graft_entry__.py` (build) first; "
                               "there is no CPU fallback")
         lib = ctypes.CDLL(LIB_PATH)
+        lenient = os.environ.get("OWL_LIB_LENIENT") == "1"  # experiments: older library builds
         for name, (res, args) in SIGNATURES.items():
+            if lenient and not hasattr(lib, name):
+                continue
             fn = getattr(lib, name)
             fn.restype = res
             fn.argtypes = args

@@ -262,7 +262,6 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     fs[i].n_warps = s.n_warps;
     fs[i].seen = seen + so;
     fs[i].walked = walked + i;
-    fs[i].perm = (const unsigned long long*)perms[i];
     fs[i].seg_index = (uint32_t)i;
     fs[i]._pad = 0;
     so += (s.n_warps + 31) / 32;
@@ -348,37 +347,47 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
         fprintf(stderr, "[owl] fold: %llu records %.3f ms pages %llu page-adds %llu claims %llu\n",
                 (unsigned long long)nrec, ms, hs.n_flush, hs.n_bypass, hs.n_claim);
         if (hs.dbg[0] | hs.dbg[1])
-          fprintf(stderr, "[owl] fold stats: fast %llu slow %llu dir_miss %llu dir_claim %llu admit %llu bcast %llu page %llu global %llu\n",
+          fprintf(stderr, "[owl] fold stats: pairs %llu general %llu pair_lead_lanes %llu pair_miss_lanes %llu single_lead_lanes %llu singles %llu s6 %llu s7 %llu\n",
                   hs.dbg[0], hs.dbg[1], hs.dbg[2], hs.dbg[3], hs.dbg[4], hs.dbg[5], hs.dbg[6], hs.dbg[7]);
       }
     }
   }
   if (status == OWL_OK) {
-    if (hs.first_error != ~0ull) {
-      const uint32_t si = (uint32_t)(hs.first_error >> 40);
-      const uint64_t idx = (hs.first_error >> 3) & ((1ull << 37) - 1); /* caller's index (the fold maps
-                                                                           bucketed records back) */
-      const uint32_t code = (uint32_t)(hs.first_error & 7);
-      status = fail(OWL_ERR_MALFORMED_TRACE, "malformed trace: run %u seq %u record %llu: %s",
-                    si < plan.size() ? plan[si].s.run : 0, si < plan.size() ? plan[si].s.seq : 0,
-                    (unsigned long long)idx, kerr_text(code));
+    /* An overflowed pass stopped early: its reports are incomplete, the regrown pass decides.  A segment that
+       is flagged warp-major but is not (a warp seen twice, or records the warp walk did not cover exactly once)
+       is reported first: walking it from the middle of a warp produces malformed-record artifacts. */
+    size_t bad_walk = plan.size();
+    for (size_t i = 0; i < plan.size() && bad_walk == plan.size(); ++i)
+      if (walked_h[i] != plan[i].s.n_records) bad_walk = i;
+    if (hs.overflow) {
     } else if (hs.not_warp_major != ~0ull) {
       const uint32_t si = (uint32_t)(hs.not_warp_major >> 32);
       status = fail(OWL_ERR_INVALID_ARG,
                     "segment (run %u, seq %u) is flagged OWL_SEG_WARP_MAJOR but warp %u's records are not contiguous",
                     plan[si].s.run, plan[si].s.seq, (uint32_t)hs.not_warp_major);
-    } else if (!hs.overflow && [&] {
-                 for (size_t i = 0; i < plan.size(); ++i)
-                   if (walked_h[i] != plan[i].s.n_records) return true;
-                 return false;
-               }()) {
-      size_t si = 0;
-      while (walked_h[si] == plan[si].s.n_records) ++si;
+    } else if (bad_walk < plan.size()) {
+      const size_t si = bad_walk;
       status = fail(OWL_ERR_INVALID_ARG,
                     "segment (run %u, seq %u) is flagged OWL_SEG_WARP_MAJOR but its records are not grouped by warp "
                     "(the warp walk covered %llu records of %llu)",
                     plan[si].s.run, plan[si].s.seq, (unsigned long long)walked_h[si],
                     (unsigned long long)plan[si].s.n_records);
+    } else if (hs.first_error != ~0ull) {
+      const uint32_t si = (uint32_t)(hs.first_error >> 40);
+      uint64_t idx = (hs.first_error >> 3) & ((1ull << 37) - 1);
+      uint32_t code = (uint32_t)(hs.first_error & 7);
+      if (si < plan.size() && perms[si]) { /* bucketed: the first bad record in the caller's order */
+        unsigned long long ic = ~0ull;
+        const cudaError_t e = owl_first_bad_record(fs[si].rec, perms[si], plan[si].s.n_records, plan[si].s.n_warps,
+                                                   &ic, st);
+        if (e == cudaSuccess && ic != ~0ull) {
+          idx = ic >> 3;
+          code = (uint32_t)(ic & 7);
+        }
+      }
+      status = fail(OWL_ERR_MALFORMED_TRACE, "malformed trace: run %u seq %u record %llu: %s",
+                    si < plan.size() ? plan[si].s.run : 0, si < plan.size() ? plan[si].s.seq : 0,
+                    (unsigned long long)idx, kerr_text(code));
     } else if (hs.limit) {
       status = (hs.limit & 2) ? fail(OWL_ERR_CAPACITY, "a traced warp visits more than %d distinct basic blocks",
                                      owl_fold_max_bbs())

@@ -77,7 +77,6 @@ struct FoldSeg {
   uint32_t* seen;     /* bitmap of n_warps bits (warp-major check), zeroed */
   unsigned long long* walked; /* records the fold walked in this segment, zeroed; = n iff every record was
                                  walked exactly once (with `seen`: the warp-major check) */
-  const unsigned long long* perm; /* channel-order segment bucketed by warp: caller's index of each record */
   uint32_t seg_index; /* position in the build's (run, seq)-sorted segment list */
   uint32_t _pad;
 };
@@ -140,6 +139,10 @@ cudaError_t owl_diff_rows(const SortedTable* A, const SortedTable* B, int ntab, 
 
 /* order-independent 128-bit fingerprint of the cells of ntab sorted tables (input-class filtering, N1) */
 cudaError_t owl_tables_fingerprint(const SortedTable* tabs, int ntab, unsigned long long fp[2], cudaStream_t st);
+
+/* the first malformed record (caller's index << 3 | KERR code, ~0 if none) of a bucketed segment */
+cudaError_t owl_first_bad_record(const uint4* rec, const uint64_t* perm, uint64_t n, uint32_t n_warps,
+                                 unsigned long long* idx_code, cudaStream_t st);
 
 /* stable bucketing of a segment's records by gwarp (channel-order input, reading R17) */
 cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, uint4* out, uint64_t* perm,

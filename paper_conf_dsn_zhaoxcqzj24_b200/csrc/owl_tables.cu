@@ -615,6 +615,49 @@ cudaError_t owl_tables_fingerprint(const SortedTable* tabs, int ntab, unsigned l
   return e;
 }
 
+namespace {
+/* Error report of a bucketed (channel-order) segment: every malformed record, by the rules of the warp walk
+   (SURVEY §8(b) conventions; the fold's slow path), mapped back to the caller's index; the minimum wins.  One
+   thread per traced warp (start detected on the gwarp change), walking it in order; records with gwarp >=
+   n_warps are checked one by one.  Only launched after a fold reported an error in such a segment. */
+__global__ void first_bad_kernel(const uint4* rec, const uint64_t* perm, uint64_t n, uint32_t n_warps,
+                                 unsigned long long* out) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t g = rec[i].z;
+    if (g >= n_warps) {
+      atomicMin(out, ((unsigned long long)perm[i] << 3) | KERR_GWARP);
+      continue;
+    }
+    if (i > 0 && rec[i - 1].z == g) continue;
+    uint32_t cur = OWL_NONE_BB;
+    for (uint64_t k = i; k < n && rec[k].z == g; ++k) {
+      const uint4 r = rec[k];
+      const uint32_t bb = (r.w >> 8) & 0x3FFFFu;
+      uint32_t code = KERR_NONE;
+      if ((r.w >> 31) == 0) {
+        if (r.x != 0 || r.y != 0 || (r.w & 0x7C0000FFu) != 0) code = KERR_BBFIELDS;
+        else cur = bb;
+      } else if ((r.y >> 28) > 8) code = KERR_MTYPE;
+      else if (cur == OWL_NONE_BB) code = KERR_NOBB;
+      else if (bb != cur) code = KERR_BBMISMATCH;
+      if (code) atomicMin(out, ((unsigned long long)perm[k] << 3) | code);
+    }
+  }
+}
+}  // namespace
+
+cudaError_t owl_first_bad_record(const uint4* rec, const uint64_t* perm, uint64_t n, uint32_t n_warps,
+                                 unsigned long long* idx_code, cudaStream_t st) {
+  unsigned long long* d = (unsigned long long*)owl_dev_alloc(8);
+  if (!d) return cudaErrorMemoryAllocation;
+  cudaError_t e = cudaMemsetAsync(d, 0xFF, 8, st);
+  if (e == cudaSuccess && n) first_bad_kernel<<<grid_for(n, 256), 256, 0, st>>>(rec, perm, n, n_warps, d);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(idx_code, d, 8, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  owl_dev_free(d);
+  return e;
+}
+
 cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, uint4* out, uint64_t* perm,
                                cudaStream_t st) {
   if (!n) return cudaSuccess;
