@@ -72,8 +72,11 @@ enum {
      per-warp program order is guaranteed (reading R17) and the library first buckets the records by
      gwarp, stably, into a scratch buffer (3x the record bytes). */
   OWL_SEG_WARP_MAJOR = 1u,
-  /* `records` is a HOST pointer (pinned or pageable).  The library streams it to the device in chunks
-     inside owl_build_adcfg (copy overlapped with the fold). */
+  /* `records` is a HOST pointer (pinned for asynchronous copies; pageable works but copies synchronously).
+     owl_build_adcfg stages host segments in waves of at most owl_config.host_chunk_bytes (a wave holds at
+     least one whole segment) through two device buffers: the copy of the next wave overlaps the fold of the
+     current one, so device memory for host records stays at 2 x the largest wave.  A channel-order host
+     segment is additionally bucketed by warp (3x its bytes of scratch until the build returns). */
   OWL_SEG_HOST_RECORDS = 2u
 };
 
@@ -99,7 +102,7 @@ typedef struct {
   uint64_t cf_capacity;     /* initial hash capacity for node / edge / triple cells (0 = auto)    */
   uint32_t max_regrow;      /* times a build may double a full table and re-run (default 6)       */
   uint32_t fold_ctas_per_sm;/* 0 = automatic                                                      */
-  uint64_t host_chunk_bytes;/* staging chunk for OWL_SEG_HOST_RECORDS (0 = 256 MiB)               */
+  uint64_t host_chunk_bytes;/* staging wave for OWL_SEG_HOST_RECORDS (0 = 256 MiB), see above        */
   uint32_t hcf_reading;     /* y-values of H_cf (SURVEY reading 5): OWL_HCF_COUNTS (0,
                                default) = joint counts c_ij; OWL_HCF_ROW_NORMALIZED (1) = the elements
                                a_ij = c_ij / x_i of the transition matrix A (Eqs. 7-8).  Other values:

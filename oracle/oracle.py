@@ -55,6 +55,8 @@ def bind(L):
     L.orc_myers.argtypes = [vp, sz, vp, sz, vp, sz]; L.orc_myers.restype = sz
     L.orc_ks_hist.argtypes = [vp, vp, sz, vp, vp, sz, ctypes.c_double, vp]; L.orc_ks_hist.restype = None
     L.orc_slots.argtypes = [vp, vp, vp, vp, sz]; L.orc_slots.restype = sz
+    L.orc_evidence_new.argtypes = [ctypes.c_uint32]; L.orc_evidence_new.restype = vp
+    L.orc_evidence_add.argtypes = [vp, ctypes.POINTER(_Seg), sz, ctypes.c_int]; L.orc_evidence_add.restype = ctypes.c_int
     return L
 
 
@@ -102,6 +104,22 @@ def build(segments, threads: int = 0) -> Adcfg:
     if not h:
         raise OracleError(lib().orc_last_error().decode())
     return Adcfg(h)
+
+
+class Evidence(Adcfg):
+    """An evidence built incrementally (O1-O4 over batches of runs merged in ascending run order): the same
+    result as build() over all the runs, for workloads larger than host memory."""
+
+    def __init__(self, input_class: int):
+        super().__init__(lib().orc_evidence_new(input_class))
+
+    def add(self, segments, threads: int = 0):
+        arr = (_Seg * max(1, len(segments)))()
+        for i, s in enumerate(segments):
+            arr[i] = _Seg(s.run, s.input_class, s.seq, s.n_warps, s.kernel_id, len(s.records),
+                          s.records.ctypes.data if len(s.records) else None)
+        if lib().orc_evidence_add(self.h, arr, len(segments), threads) != 0:
+            raise OracleError(lib().orc_last_error().decode())
 
 
 def _rows(fn, dtype, *args):

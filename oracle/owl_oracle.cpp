@@ -96,6 +96,7 @@ struct Adcfg {
   std::map<K3, uint64_t> edge;
   std::map<K4, uint64_t> triple;
   std::map<K5, uint64_t> addr;
+  uint32_t max_run = 0; /* incremental builds: the last run merged */
 };
 
 struct BadRecord {
@@ -406,6 +407,70 @@ void* orc_build(const orc_segment* segs, size_t n_segs, int threads) {
   }
   if (per.empty()) ev->n_runs = 0;
   return ev;
+}
+
+/* Incremental form of orc_build for workloads larger than host memory (the full-size parity digests): an
+   evidence starts empty; each orc_evidence_add builds the per-run A-DCFGs of a batch of runs (O1-O3, thread
+   pool) and merges them into the evidence in ascending run order (O4), exactly as orc_build would after the
+   runs already added.  Batches must hold runs above every run added before.  Returns 0, or -1 on a malformed
+   trace or an out-of-order run (message in orc_last_error()). */
+void* orc_evidence_new(uint32_t input_class) {
+  Adcfg* ev = new Adcfg();
+  ev->input_class = input_class;
+  ev->n_runs = 0;
+  return ev;
+}
+
+int orc_evidence_add(void* h, const orc_segment* segs, size_t n_segs, int threads) {
+  Adcfg* ev = (Adcfg*)h;
+  std::map<uint32_t, std::vector<const orc_segment*>> runs;
+  for (size_t i = 0; i < n_segs; ++i) runs[segs[i].run].push_back(&segs[i]);
+  if (!runs.empty() && ev->n_runs > 0 && !(runs.begin()->first > ev->max_run)) {
+    g_err = "orc_evidence_add: runs must be added in ascending order";
+    return -1;
+  }
+  std::vector<uint32_t> run_ids;
+  for (auto& r : runs) {
+    std::sort(r.second.begin(), r.second.end(),
+              [](const orc_segment* a, const orc_segment* b) { return a->seq < b->seq; });
+    run_ids.push_back(r.first);
+  }
+  std::vector<Adcfg> per(run_ids.size());
+  std::vector<BadRecord> bads(run_ids.size());
+  std::atomic<size_t> next(0);
+  int nt = threads > 0 ? threads : (int)std::max(1u, std::thread::hardware_concurrency());
+  if ((size_t)nt > run_ids.size()) nt = (int)std::max<size_t>(1, run_ids.size());
+  auto worker = [&]() {
+    for (;;) {
+      size_t i = next.fetch_add(1);
+      if (i >= run_ids.size()) break;
+      build_run(runs[run_ids[i]], per[i], bads[i]);
+    }
+  };
+  std::vector<std::thread> pool;
+  for (int t = 1; t < nt; ++t) pool.emplace_back(worker);
+  worker();
+  for (auto& t : pool) t.join();
+  BadRecord bad;
+  for (auto& b : bads) if (b.any) bad.note(b.run, b.seq, b.index, b.why.c_str());
+  if (bad.any) {
+    char buf[256];
+    snprintf(buf, sizeof buf, "malformed trace: run %u seq %u record %llu: %s", bad.run, bad.seq,
+             (unsigned long long)bad.index, bad.why.c_str());
+    g_err = buf;
+    return -1;
+  }
+  for (size_t i = 0; i < per.size(); ++i) { /* O4 in ascending run order; the first run of all starts the evidence */
+    if (ev->n_runs == 0) {
+      const uint32_t cls = ev->input_class;
+      *ev = std::move(per[i]);
+      ev->input_class = cls;
+    } else {
+      merge_run(*ev, per[i]);
+    }
+    ev->max_run = run_ids[i];
+  }
+  return 0;
 }
 
 /* Bad record location of the last failed orc_build: run, seq, index (for parity of error reports). */

@@ -874,7 +874,6 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
 }  // namespace
 
 int owl_fold_ctas_per_sm() { return 1; }
-int owl_fold_runs_per_warp() { return 1; }
 size_t owl_fold_scratch_bytes(int grid) { return (size_t)grid * FOLD_WARPS * 2 * VCAP * sizeof(uint32_t); }
 int owl_fold_max_bbs() { return 32 + VCAP; }
 

@@ -74,6 +74,7 @@ struct owl_ctx {
   std::map<uint32_t, RemoteRun> remote;
   FoldStatus* d_status = nullptr;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  cudaStream_t copy_stream = nullptr; /* host-record staging (fold_pass) */
   uint64_t cap_hint[T_NUM] = {0, 0, 0, 0};
   /* stats */
   uint64_t fold_launches = 0;
@@ -212,7 +213,13 @@ const char* kerr_text(uint32_t code) {
 }
 
 /* One fold pass over the planned segments into `tab` (A1-A3).  Returns OWL_OK, or an error; sets
-   *overflow to the bitmask of tables that must grow. */
+   *overflow to the bitmask of tables that must grow.
+
+   Device-resident segments are folded in one launch.  Host segments (OWL_SEG_HOST_RECORDS) are staged in waves
+   of at most host_chunk_bytes (a wave holds at least one segment) through two device buffers: the copy of wave
+   k + 1 (copy stream) overlaps the fold of wave k (context stream), and a buffer is refilled only after the fold
+   that read it.  Channel-order segments are bucketed by warp on the device first (3x their bytes of scratch,
+   held until the pass returns: the error report of a malformed record maps it back through the permutation). */
 owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable* tab, unsigned* overflow,
                      uint64_t* n_records) {
   const cudaStream_t st = ctx->stream;
@@ -221,7 +228,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
   std::vector<FoldSeg> fs(plan.size());
   std::vector<void*> scratch;
   std::vector<uint64_t*> perms(plan.size(), nullptr);
-  uint64_t seen_words = 0, tiles = 0, nrec = 0;
+  uint64_t seen_words = 0, nrec = 0;
   for (size_t i = 0; i < plan.size(); ++i) seen_words += (plan[i].s.n_warps + 31) / 32;
   uint32_t* seen = (uint32_t*)owl_dev_alloc((seen_words + 1) * 4);
   if (!seen) return fail(OWL_ERR_OUT_OF_MEMORY, "fold: warp bitmap");
@@ -231,33 +238,15 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
   if (!walked) { owl_dev_free(seen); return fail(OWL_ERR_OUT_OF_MEMORY, "fold: walk counters"); }
   scratch.push_back(walked);
   CUDA_TRY(cudaMemsetAsync(walked, 0, (plan.size() + 1) * 8, st), "fold: memset");
-  uint64_t so = 0;
-  owl_status status = OWL_OK;
-  for (size_t i = 0; i < plan.size() && status == OWL_OK; ++i) {
+  /* launches: device segments, then waves of host segments */
+  const uint64_t chunk = ctx->cfg.host_chunk_bytes ? ctx->cfg.host_chunk_bytes : (256ull << 20);
+  std::vector<std::vector<size_t>> launches(1);
+  std::vector<uint64_t> wave_bytes(1, 0);
+  for (size_t i = 0, so = 0; i < plan.size(); ++i) {
     const owl_segment& s = plan[i].s;
-    const uint4* rec = (const uint4*)s.records;
-    if (s.n_records && (s.flags & OWL_SEG_HOST_RECORDS)) { /* stage host records into HBM */
-      uint4* d = (uint4*)owl_dev_alloc(s.n_records * 16);
-      if (!d) { status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: staging %llu records", (unsigned long long)s.n_records); break; }
-      scratch.push_back(d);
-      cudaError_t e = cudaMemcpyAsync(d, s.records, s.n_records * 16, cudaMemcpyHostToDevice, st);
-      if (e != cudaSuccess) { status = cuda_fail(e, "fold: H2D"); break; }
-      rec = d;
-    }
-    if (s.n_records && !(s.flags & OWL_SEG_WARP_MAJOR)) { /* channel order: stable bucket by warp (R17) */
-      uint4* d = (uint4*)owl_dev_alloc(s.n_records * 16);
-      uint64_t* perm = (uint64_t*)owl_dev_alloc(s.n_records * 8);
-      if (!d || !perm) { owl_dev_free(d); owl_dev_free(perm); status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: bucketing"); break; }
-      scratch.push_back(d);
-      scratch.push_back(perm);
-      cudaError_t e = owl_bucket_by_warp(rec, s.n_records, s.n_warps, d, perm, st);
-      if (e != cudaSuccess) { status = cuda_fail(e, "fold: bucketing"); break; }
-      rec = d;
-      perms[i] = perm;
-    }
-    fs[i].rec = rec;
+    fs[i].rec = (const uint4*)s.records;
     fs[i].n = s.n_records;
-    fs[i].tile0 = tiles;
+    fs[i].tile0 = 0;
     fs[i].slot = plan[i].slot;
     fs[i].n_warps = s.n_warps;
     fs[i].seen = seen + so;
@@ -265,56 +254,121 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     fs[i].seg_index = (uint32_t)i;
     fs[i]._pad = 0;
     so += (s.n_warps + 31) / 32;
-    tiles += (s.n_records + (1ull << tile_shift) - 1) >> tile_shift;
     nrec += s.n_records;
-  }
-  /* run batching (owl_fold.cu): groups of up to owl_fold_runs_per_warp() segments of one slot, ascending run;
-     one warp walks all members of a group at the same tile position */
-  const size_t group_max = (size_t)owl_fold_runs_per_warp();
-  std::vector<uint32_t> order(fs.size());
-  for (size_t i = 0; i < order.size(); ++i) order[i] = (uint32_t)i;
-  std::stable_sort(order.begin(), order.end(), [&](uint32_t x, uint32_t y) { return fs[x].slot < fs[y].slot; });
-  std::vector<FoldSeg> gsegs;
-  std::vector<FoldGroup> groups;
-  uint64_t items = 0;
-  for (size_t i = 0; i < order.size();) {
-    size_t e = i;
-    uint64_t npos = 0;
-    while (e < order.size() && e - i < group_max && fs[order[e]].slot == fs[order[i]].slot) {
-      npos = std::max<uint64_t>(npos, (fs[order[e]].n + (1ull << tile_shift) - 1) >> tile_shift);
-      ++e;
+    if (!(s.flags & OWL_SEG_HOST_RECORDS) || !s.n_records) {
+      launches[0].push_back(i);
+      continue;
     }
-    FoldGroup g;
-    g.item0 = items;
-    g.first_seg = (uint32_t)gsegs.size();
-    g.n_members = (uint32_t)(e - i);
-    for (size_t q = i; q < e; ++q) gsegs.push_back(fs[order[q]]);
-    if (npos) { groups.push_back(g); items += npos; }
-    else gsegs.resize(g.first_seg);
-    i = e;
+    const uint64_t b = s.n_records * 16;
+    if (launches.size() == 1 || (wave_bytes.back() && wave_bytes.back() + b > chunk)) {
+      launches.emplace_back();
+      wave_bytes.push_back(0);
+    }
+    launches.back().push_back(i);
+    wave_bytes.back() += b;
   }
-  FoldSeg* dsegs = nullptr;
-  FoldGroup* dgroups = nullptr;
-  if (status == OWL_OK) {
-    dsegs = (FoldSeg*)owl_dev_alloc(gsegs.size() * sizeof(FoldSeg) + 16);
-    dgroups = (FoldGroup*)owl_dev_alloc(groups.size() * sizeof(FoldGroup) + 16);
-    if (!dsegs || !dgroups) status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: segment table");
+  uint64_t stage_cap = 0;
+  for (size_t w = 1; w < wave_bytes.size(); ++w) stage_cap = std::max(stage_cap, wave_bytes[w]);
+  uint4* stage[2] = {nullptr, nullptr};
+  cudaEvent_t ready[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr};
+  owl_status status = OWL_OK;
+  if (stage_cap) {
+    for (int k = 0; k < 2 && k + 1 < (int)launches.size(); ++k) {
+      stage[k] = (uint4*)owl_dev_alloc(stage_cap);
+      if (!stage[k]) status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: host staging buffers (2 x %llu bytes)",
+                                   (unsigned long long)stage_cap);
+      else scratch.push_back(stage[k]);
+      cudaEventCreateWithFlags(&ready[k], cudaEventDisableTiming);
+      cudaEventCreateWithFlags(&freed[k], cudaEventDisableTiming);
+    }
+    if (!ctx->copy_stream) cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking);
   }
+  const int per_sm = ctx->cfg.fold_ctas_per_sm ? (int)ctx->cfg.fold_ctas_per_sm : owl_fold_ctas_per_sm();
+  const int grid = ctx->n_sm * per_sm;
+  uint32_t* vmap = status == OWL_OK ? (uint32_t*)owl_dev_alloc(owl_fold_scratch_bytes(grid)) : nullptr;
+  if (status == OWL_OK && !vmap) status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: visit-map scratch");
+  if (vmap) scratch.push_back(vmap);
   FoldStatus hs;
+  hs.first_error = ~0ull;
+  hs.not_warp_major = ~0ull;
+  hs.overflow = 0;
+  hs.limit = 0;
+  hs.tile_counter = 0;
+  hs.n_flush = hs.n_bypass = hs.n_claim = 0;
+  for (int i = 0; i < 8; ++i) hs.dbg[i] = 0;
+  if (status == OWL_OK) cudaMemcpyAsync(ctx->d_status, &hs, sizeof hs, cudaMemcpyHostToDevice, st);
   std::vector<unsigned long long> walked_h(plan.size(), 0);
-  if (status == OWL_OK) {
+  float fold_ms = 0;
+  uint64_t launched = 0;
+  auto stage_wave = [&](size_t w) -> cudaError_t { /* copy stream: wave w into stage[(w - 1) % 2] */
+    const int k = (int)((w - 1) & 1);
+    cudaError_t e = cudaStreamWaitEvent(ctx->copy_stream, freed[k], 0);
+    uint64_t off = 0;
+    for (size_t i : launches[w]) {
+      const owl_segment& s = plan[i].s;
+      if (e == cudaSuccess)
+        e = cudaMemcpyAsync(stage[k] + off, s.records, s.n_records * 16, cudaMemcpyHostToDevice, ctx->copy_stream);
+      fs[i].rec = stage[k] + off;
+      off += s.n_records;
+    }
+    if (e == cudaSuccess) e = cudaEventRecord(ready[k], ctx->copy_stream);
+    return e;
+  };
+  for (int k = 0; k < 2; ++k)
+    if (freed[k]) cudaEventRecord(freed[k], st);
+  if (status == OWL_OK && launches.size() > 1) {
+    const cudaError_t e = stage_wave(1);
+    if (e != cudaSuccess) status = cuda_fail(e, "fold: H2D staging");
+  }
+  for (size_t w = 0; w < launches.size() && status == OWL_OK; ++w) {
+    if (w + 1 < launches.size() && w >= 1) { /* prefetch the next wave while this one is folded */
+      const cudaError_t e = stage_wave(w + 1);
+      if (e != cudaSuccess) { status = cuda_fail(e, "fold: H2D staging"); break; }
+    }
+    if (w >= 1) cudaStreamWaitEvent(st, ready[(w - 1) & 1], 0);
+    /* channel order: stable bucket by warp (R17) */
+    for (size_t i : launches[w]) {
+      const owl_segment& s = plan[i].s;
+      if (!s.n_records || (s.flags & OWL_SEG_WARP_MAJOR)) continue;
+      uint4* d = (uint4*)owl_dev_alloc(s.n_records * 16);
+      uint64_t* perm = (uint64_t*)owl_dev_alloc(s.n_records * 8);
+      if (!d || !perm) { owl_dev_free(d); owl_dev_free(perm); status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: bucketing"); break; }
+      scratch.push_back(d);
+      scratch.push_back(perm);
+      cudaError_t e = owl_bucket_by_warp(fs[i].rec, s.n_records, s.n_warps, d, perm, st);
+      if (e != cudaSuccess) { status = cuda_fail(e, "fold: bucketing"); break; }
+      fs[i].rec = d;
+      perms[i] = perm;
+    }
+    if (status != OWL_OK) break;
+    /* work items: (segment, tile of 2^tile_shift records), one range per segment */
+    std::vector<FoldSeg> lsegs;
+    std::vector<FoldGroup> groups;
+    uint64_t items = 0, lrec = 0;
+    for (size_t i : launches[w]) {
+      const uint64_t ntile = (fs[i].n + (1ull << tile_shift) - 1) >> tile_shift;
+      if (!ntile) continue;
+      FoldGroup g;
+      g.item0 = items;
+      g.first_seg = (uint32_t)lsegs.size();
+      g._pad = 0;
+      lsegs.push_back(fs[i]);
+      groups.push_back(g);
+      items += ntile;
+      lrec += fs[i].n;
+    }
+    if (!items) {
+      if (w >= 1) cudaEventRecord(freed[(w - 1) & 1], st);
+      continue;
+    }
+    FoldSeg* dsegs = (FoldSeg*)owl_dev_alloc(lsegs.size() * sizeof(FoldSeg) + 16);
+    FoldGroup* dgroups = (FoldGroup*)owl_dev_alloc(groups.size() * sizeof(FoldGroup) + 16);
+    if (!dsegs || !dgroups) { owl_dev_free(dsegs); owl_dev_free(dgroups); status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: segment table"); break; }
     scratch.push_back(dsegs);
     scratch.push_back(dgroups);
-    cudaMemcpyAsync(dsegs, gsegs.data(), gsegs.size() * sizeof(FoldSeg), cudaMemcpyHostToDevice, st);
+    cudaMemcpyAsync(dsegs, lsegs.data(), lsegs.size() * sizeof(FoldSeg), cudaMemcpyHostToDevice, st);
     cudaMemcpyAsync(dgroups, groups.data(), groups.size() * sizeof(FoldGroup), cudaMemcpyHostToDevice, st);
-    hs.first_error = ~0ull;
-    hs.not_warp_major = ~0ull;
-    hs.overflow = 0;
-    hs.limit = 0;
-    hs.tile_counter = 0;
-    hs.n_flush = hs.n_bypass = hs.n_claim = 0;
-    for (int i = 0; i < 8; ++i) hs.dbg[i] = 0;
-    cudaMemcpyAsync(ctx->d_status, &hs, sizeof hs, cudaMemcpyHostToDevice, st);
+    cudaMemsetAsync(&ctx->d_status->tile_counter, 0, sizeof(unsigned long long), st); /* the launch's work counter */
     FoldArgs a;
     a.segs = dsegs;
     a.groups = dgroups;
@@ -324,32 +378,49 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     for (int t = 0; t < T_NUM; ++t) a.tab[t] = tab[t];
     a.status = ctx->d_status;
     a.mode = getenv("OWL_FOLD_MODE") ? (uint32_t)atoi(getenv("OWL_FOLD_MODE")) : 0u;
-    const int per_sm = ctx->cfg.fold_ctas_per_sm ? (int)ctx->cfg.fold_ctas_per_sm : owl_fold_ctas_per_sm();
-    const int grid = ctx->n_sm * per_sm;
-    a.vmap = (uint32_t*)owl_dev_alloc(owl_fold_scratch_bytes(grid));
-    scratch.push_back(a.vmap);
+    a.vmap = vmap;
     cudaEventRecord(ctx->ev0, st);
-    cudaError_t e = !a.vmap ? cudaErrorMemoryAllocation : items ? owl_launch_fold(a, grid, st) : cudaSuccess;
+    cudaError_t e = owl_launch_fold(a, grid, st);
     cudaEventRecord(ctx->ev1, st);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(&hs, ctx->d_status, sizeof hs, cudaMemcpyDeviceToHost, st);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(walked_h.data(), walked, plan.size() * 8, cudaMemcpyDeviceToHost, st);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-    if (e != cudaSuccess) status = cuda_fail(e, "fold kernel");
-    else {
+    if (w >= 1) cudaEventRecord(freed[(w - 1) & 1], st);
+    if (e == cudaSuccess && launches.size() > 1) e = cudaEventSynchronize(ctx->ev1); /* per-launch timing */
+    if (e != cudaSuccess) { status = cuda_fail(e, "fold kernel"); break; }
+    if (launches.size() > 1) {
       float ms = 0;
       cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1);
-      if (items) ctx->fold_launches += 1;
-      ctx->last_fold_ms = ms;
-      ctx->last_fold_records = nrec;
-      ctx->total_fold_ms += ms;
-      ctx->total_fold_records += nrec;
-      if (getenv("OWL_FOLD_VERBOSE")) {
-        fprintf(stderr, "[owl] fold: %llu records %.3f ms pages %llu page-adds %llu claims %llu\n",
-                (unsigned long long)nrec, ms, hs.n_flush, hs.n_bypass, hs.n_claim);
-        if (hs.dbg[0] | hs.dbg[1])
-          fprintf(stderr, "[owl] fold stats: pairs %llu general %llu pair_lead_lanes %llu pair_miss_lanes %llu single_lead_lanes %llu singles %llu s6 %llu s7 %llu\n",
-                  hs.dbg[0], hs.dbg[1], hs.dbg[2], hs.dbg[3], hs.dbg[4], hs.dbg[5], hs.dbg[6], hs.dbg[7]);
-      }
+      fold_ms += ms;
+    }
+    ++launched;
+    (void)lrec;
+  }
+  cudaError_t e = status == OWL_OK ? cudaMemcpyAsync(&hs, ctx->d_status, sizeof hs, cudaMemcpyDeviceToHost, st)
+                                   : cudaSuccess;
+  if (status == OWL_OK && e == cudaSuccess)
+    e = cudaMemcpyAsync(walked_h.data(), walked, plan.size() * 8, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (ctx->copy_stream) cudaStreamSynchronize(ctx->copy_stream);
+  for (int k = 0; k < 2; ++k) {
+    if (ready[k]) cudaEventDestroy(ready[k]);
+    if (freed[k]) cudaEventDestroy(freed[k]);
+  }
+  if (status == OWL_OK && e != cudaSuccess) status = cuda_fail(e, "fold kernel");
+  if (status == OWL_OK) {
+    if (launches.size() == 1) {
+      float ms = 0;
+      if (launched) cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1);
+      fold_ms = ms;
+    }
+    ctx->fold_launches += launched;
+    ctx->last_fold_ms = fold_ms;
+    ctx->last_fold_records = nrec;
+    ctx->total_fold_ms += fold_ms;
+    ctx->total_fold_records += nrec;
+    if (getenv("OWL_FOLD_VERBOSE")) {
+      fprintf(stderr, "[owl] fold: %llu records %.3f ms pages %llu page-adds %llu claims %llu (%llu launches)\n",
+              (unsigned long long)nrec, fold_ms, hs.n_flush, hs.n_bypass, hs.n_claim, (unsigned long long)launched);
+      if (hs.dbg[0] | hs.dbg[1])
+        fprintf(stderr, "[owl] fold stats: fast %llu slow %llu %llu %llu %llu %llu %llu %llu\n", hs.dbg[0],
+                hs.dbg[1], hs.dbg[2], hs.dbg[3], hs.dbg[4], hs.dbg[5], hs.dbg[6], hs.dbg[7]);
     }
   }
   if (status == OWL_OK) {
@@ -533,6 +604,7 @@ OWL_API owl_status owl_ctx_destroy(owl_ctx* ctx) {
   owl_dev_trim(ctx->device);
   if (ctx->ev0) cudaEventDestroy(ctx->ev0);
   if (ctx->ev1) cudaEventDestroy(ctx->ev1);
+  if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
   delete ctx;
   return OWL_OK;
 }

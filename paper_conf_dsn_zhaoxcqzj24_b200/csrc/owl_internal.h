@@ -81,12 +81,12 @@ struct FoldSeg {
   uint32_t _pad;
 };
 
-/* A work item of the fold is (group, tile position p): one warp folds tile p of every segment of the group
-   at once.  Groups hold up to owl_fold_runs_per_warp() segments of one slot (run batching). */
+/* A work item of the fold is (segment, tile position p): one warp folds the traced warps starting in tile p.
+   The items of segment first_seg are item0 .. item0 + its number of tiles - 1. */
 struct FoldGroup {
-  uint64_t item0;     /* first work-item id of this group */
-  uint32_t first_seg; /* index of its first member in FoldArgs::segs */
-  uint32_t n_members;
+  uint64_t item0;     /* first work-item id of the segment */
+  uint32_t first_seg; /* the segment's index in FoldArgs::segs */
+  uint32_t _pad;
 };
 
 struct FoldArgs {
@@ -104,7 +104,6 @@ struct FoldArgs {
 /* ---- launchers (owl_fold.cu, owl_tables.cu, owl_ks.cu, owl_exchange.cu) ---- */
 cudaError_t owl_launch_fold(const FoldArgs& a, int grid, cudaStream_t st);
 int owl_fold_ctas_per_sm();
-int owl_fold_runs_per_warp();
 size_t owl_fold_scratch_bytes(int grid);
 int owl_fold_max_bbs(); /* distinct BBs one traced warp may visit */
 

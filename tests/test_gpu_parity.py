@@ -508,9 +508,13 @@ def test_channel_order_first_bad_record(ctx):
         ctx.forget_runs([0])
 
 
-@pytest.mark.parametrize("cfg,div,interleaved", [(2, 32, False), (5, 32, True), (4, 256, False)])
-def test_host_records_e2e_path(ctx, cfg, div, interleaved):
-    """OWL_SEG_HOST_RECORDS (the bench's e2e leg): host buffers staged by the library give the oracle's result."""
+@pytest.mark.parametrize("cfg,div,interleaved,chunk", [(2, 32, False, 0), (5, 32, True, 0), (4, 256, False, 0),
+                                                       (2, 32, False, 1 << 20), (5, 32, True, 1 << 20),
+                                                       (9, 16, False, 3 << 20)])
+def test_host_records_e2e_path(ctx, cfg, div, interleaved, chunk):
+    """OWL_SEG_HOST_RECORDS (the bench's e2e leg): host buffers staged by the library give the oracle's result,
+    in one wave or (small host_chunk_bytes) in many waves through the two staging buffers."""
+    ctx.set_config(host_chunk_bytes=chunk)
     p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=2, runs_rnd=2)
     runs = list(range(p.n_runs))
     segs = []
@@ -523,11 +527,15 @@ def test_host_records_e2e_path(ctx, cfg, div, interleaved):
             flags = api.OWL_SEG_HOST_RECORDS | (0 if interleaved else api.OWL_SEG_WARP_MAJOR)
             segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, host, len(rec), flags=flags))
     ctx.ingest(segs)
+    ctx.reset_stats()
     try:
         ef, er = ctx.build(_runs_of(p, 0)), ctx.build(_runs_of(p, 1))
         osg = _oracle_segments(p, runs)
         of, orr = oracle.build(osg[0]), oracle.build(osg[1])
         assert ef.export() == of.export() and er.export() == orr.export()
         assert_leak_parity(ctx.leak_test(ef, er, SIG), oracle.leak_test(of, orr, SIG))
+        if chunk:
+            assert ctx.stats()["fold_launches"] > 2  # several waves
     finally:
         ctx.forget_runs(runs)
+        ctx.set_config()
