@@ -266,6 +266,17 @@ def e2e_leg(args, p, api, tracegen, dev, stream, n_runs_e2e, my_runs, world=1, r
                       f"memory, {steps} steps"}
 
 
+def _chunks(tracegen, p, runs, budget_bytes):
+    """Contiguous blocks of the (ascending) runs whose records fit in `budget_bytes` of HBM at once (record sizes
+    estimated from the first runs; exactness never depends on the split)."""
+    if not runs:
+        return []
+    sample = runs[:2]
+    per_run = 16 * sum(tracegen.host_count(p, r, m.seq) for r in sample for m in tracegen.run_segments(p, r)) / len(sample)
+    k = max(1, int(budget_bytes // max(per_run, 1.0)))
+    return [runs[i:i + k] for i in range(0, len(runs), k)]
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -283,30 +294,49 @@ def run_ours(args):
         if share:
             dist.init_process_group("gloo")
         else:
+            os.environ.setdefault("NCCL_DEBUG", "INFO")  # the driver checks comm_nranks in the log
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     cfg = args.config
     base = tracegen.Params.preset(cfg)
-    # weak scaling: each rank holds the full per-GPU workload's runs (global run ids are disjoint)
-    rpr = base.n_runs
-    p = tracegen.Params.preset(cfg, runs_fix=base.runs_fix * world, runs_rnd=base.runs_rnd * world)
-    my_runs = list(range(rank * rpr, (rank + 1) * rpr))
+    # scaling: weak (default: every rank holds the full per-GPU workload of its own runs) or strong (C5, the north
+    # star's scaling sweep: the paper-size run set is split across the ranks)
+    strong = args.scaling == "strong" or (args.scaling == "auto" and cfg == 5)
+    if strong:
+        p = base
+        from paper_conf_dsn_zhaoxcqzj24_b200 import dist as D
+        my_runs = D.shard(list(range(p.n_runs)), world, rank) if world > 1 else list(range(p.n_runs))
+    else:
+        rpr = base.n_runs
+        p = tracegen.Params.preset(cfg, runs_fix=base.runs_fix * world, runs_rnd=base.runs_rnd * world)
+        my_runs = list(range(rank * rpr, (rank + 1) * rpr))
     if args.runs:
         my_runs = my_runs[: args.runs]
     ctx = api.Context(local)
     stream = torch.cuda.current_stream(dev)
-    segs = []
+    chunks = _chunks(tracegen, p, my_runs, args.hbm_budget_gb * 1e9)
+    resident = len(chunks) == 1
+    if not resident and world > 1:
+        raise SystemExit("bench: a rank's runs exceed --hbm-budget-gb; use more GPUs or strong scaling")
+
+    def generate(runs):
+        segs = []
+        for r in runs:
+            for m in tracegen.run_segments(p, r):
+                buf, n = tracegen.device_records(p, r, m.seq, device=dev, stream=stream)
+                segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, n))
+        torch.cuda.synchronize()
+        return segs
+
     t_gen = time.perf_counter()
-    for r in my_runs:
-        for m in tracegen.run_segments(p, r):
-            buf, n = tracegen.device_records(p, r, m.seq, device=dev, stream=stream)
-            segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, n))
-    torch.cuda.synchronize()
+    segs = generate(chunks[0]) if chunks else []
     t_gen = time.perf_counter() - t_gen
     n_records = sum(s.n_records for s in segs)
+    if not resident:
+        for c in chunks[1:]:
+            n_records += sum(tracegen.host_count(p, r, m.seq) for r in c for m in tracegen.run_segments(p, r))
     ctx.ingest(segs, stream)
-    all_runs = list(range(p.n_runs))
     if world > 1:
         # §8(e): slot agreement over all runs, then every step folds this rank's shard into partial evidences
         # and exchanges cells by owner (paper_conf_dsn_zhaoxcqzj24_b200/dist.py)
@@ -315,12 +345,13 @@ def run_ours(args):
         all_meta = D.gather_sequences(meta)
         D.agree_slots(ctx, all_meta, my_runs)
         all_runs = sorted(all_meta)
-        rf, rr = _class_runs(p, all_runs, 0), _class_runs(p, all_runs, 1)
     else:
-        rf, rr = _class_runs(p, my_runs, 0), _class_runs(p, my_runs, 1)
+        all_runs = list(my_runs)
+    rf_all, rr_all = _class_runs(p, all_runs, 0), _class_runs(p, all_runs, 1)
 
     out = {}
     brk = {}
+    timed_ms = [0.0]
 
     def tick(name, t0):
         if args.breakdown:
@@ -330,13 +361,8 @@ def run_ours(args):
             return t1
         return t0
 
-    def step():
+    def analysis(ef, er, held):
         t0 = time.perf_counter()
-        ef = ctx.build(rf)
-        t0 = tick("build_fix", t0)
-        er = ctx.build(rr)
-        t0 = tick("build_rnd", t0)
-        held = [ef, er]
         if world > 1:  # the one exchange: partial evidences -> owners' evidences
             (ef, bf), (er, br) = D.owner_evidence(ctx, ef, world, rank), D.owner_evidence(ctx, er, world, rank)
             held += [ef, er]
@@ -348,11 +374,60 @@ def run_ours(args):
             d = ctx.diff(ef, er)
             t0 = tick("diff", t0)
             lk = ctx.leak_test(ef, er, 0.05)
-        t0 = tick("leak_test", t0)
+        tick("leak_test", t0)
         out.update(n_diff=len(d), n_leaks=len(lk), info_f=ef.info(), info_r=er.info())
+
+    def step():
+        if resident:
+            t0 = time.perf_counter()
+            ef = ctx.build(rf_all)
+            t0 = tick("build_fix", t0)
+            er = ctx.build(rr_all)
+            tick("build_rnd", t0)
+            held = [ef, er]
+            analysis(ef, er, held)
+            for g in held:
+                g.destroy()
+            return
+        # chunked (the workload exceeds one GPU's HBM): each chunk's records are generated (untimed), then
+        # folded and merged into the evidences (timed, CUDA events); the analysis is timed
+        nonlocal segs
+        ev = {0: None, 1: None}
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        for ci, c in enumerate(chunks):
+            if ci > 0 or segs is None:
+                ctx.forget_runs([r for r in my_runs if r not in c])
+                segs = None
+                torch.cuda.empty_cache()
+                segs = generate(c)
+                ctx.ingest(segs, stream)
+            e0.record(stream)
+            cset = set(c)
+            for cls, allc in ((0, rf_all), (1, rr_all)):
+                mine = [r for r in allc if r in cset]
+                if not mine:
+                    continue
+                if ev[cls] is None:
+                    ev[cls] = ctx.build(mine)
+                else:
+                    ev[cls].accumulate(mine)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            timed_ms[0] += e0.elapsed_time(e1)
+        e0.record(stream)
+        held = [ev[0], ev[1]]
+        analysis(ev[0], ev[1], held)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        timed_ms[0] += e0.elapsed_time(e1)
         for g in held:
             g.destroy()
-        tick("destroy", t0)
+        # the next step starts from the first chunk again
+        ctx.forget_runs(my_runs)
+        segs = None
+        torch.cuda.empty_cache()
+        segs = generate(chunks[0])
+        ctx.ingest(segs, stream)
 
     clocks = ClockSampler(local)
     clocks.start()  # nvidia-smi starts up during the warm-up; only timed-region samples are kept
@@ -360,6 +435,7 @@ def run_ours(args):
         step()
     brk.clear()
     ctx.reset_stats()
+    timed_ms[0] = 0.0
     clocks.wait_ready()
     if world > 1:
         dist.barrier()
@@ -372,29 +448,39 @@ def run_ours(args):
     e1.record(stream)
     torch.cuda.synchronize()
     ck = clocks.stop()
-    ms = e0.elapsed_time(e1) / args.steps
+    ms = (e0.elapsed_time(e1) if resident else timed_ms[0]) / args.steps
     st = ctx.stats()
     if world > 1:
         t = torch.tensor([ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
-    total_records = n_records * world
+        t = torch.tensor([float(n_records)], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        total_records = int(t.item())
+    else:
+        total_records = n_records
     value = total_records / (ms / 1e3)
     peak, peak_src = _peaks()
     fold_ms = st["total_fold_ms"] / max(1, st["fold_launches"])
     fold_bytes = 16.0 * st["total_fold_records"] / max(1, st["fold_launches"])
     achieved = fold_bytes / (fold_ms / 1e3) / 1e9
+    mode = "strong" if strong else "weak"
     res = {
         "metric": METRIC, "value": value, "unit": "records/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": mode,
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-        "config": {"workload": tracegen.CONFIG_NAMES[cfg], "runs_per_gpu": len(my_runs),
+        "config": {"workload": tracegen.CONFIG_NAMES[cfg], "runs_per_gpu": len(my_runs), "runs_total": p.n_runs,
                    "records_per_gpu": n_records, "bytes_per_gpu": 16 * n_records,
                    "l2": "inputs (%.1f GB) >> 126 MB L2; no flush needed" % (16 * n_records / 1e9),
-                   "parallelism": f"dp{world} (runs sharded, key-hash exchange)" if world > 1 else "single GPU",
+                   "parallelism": f"dp{world} (runs sharded, key-hash exchange, {mode} scaling)" if world > 1
+                   else "single GPU",
+                   "hbm_chunks": len(chunks),
+                   "timing": "whole steps, CUDA events" if resident else
+                   f"{len(chunks)} chunks per step: each chunk's on-device generation untimed, its fold + merge and "
+                   "the analysis timed with CUDA events",
                    "generate_s_untimed": round(t_gen, 2)},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": _traffic(fold_bytes / 16.0), "kernel": "fold_kernel",
+                     "traffic": _traffic(fold_bytes / 16.0) if cfg == 2 else None, "kernel": "fold_kernel",
                      "note": f"16 B/record algorithmic; {st['fold_launches']} fold launches, "
                              f"{fold_ms:.2f} ms avg (CUDA events on the launch stream); peak {peak_src}"},
         "clocks": ck,
@@ -403,14 +489,19 @@ def run_ours(args):
         "result": {"n_diff_rows": out.get("n_diff"), "n_leaks": out.get("n_leaks"),
                    "cells_fix": out.get("info_f", {}).get("n_cells"), "cells_rnd": out.get("info_r", {}).get("n_cells")},
     }
-    n_launch, names = count_launches(step)
-    res["gpu_launches"] = n_launch * args.steps
-    res["gpu_launches_per_step"] = names
+    if resident:
+        n_launch, names = count_launches(step)
+        res["gpu_launches"] = n_launch * args.steps
+        res["gpu_launches_per_step"] = names
+    else:
+        res["gpu_launches"] = None
     if not args.no_e2e:
         del segs
         ctx.forget_runs(my_runs)
         torch.cuda.empty_cache()
-        res["e2e"] = e2e_leg(args, p, api, tracegen, dev, stream, args.e2e_runs, my_runs, world, rank)
+        per_run = 16 * n_records / max(1, len(my_runs))
+        e2e_runs = max(2, min(args.e2e_runs, int(args.e2e_gb * 1e9 // max(per_run, 1)) // 2 * 2))
+        res["e2e"] = e2e_leg(args, p, api, tracegen, dev, stream, e2e_runs, my_runs, world, rank)
     if rank == 0 and not args.no_cpu:
         res["cpu_baseline"] = cpu_baseline(cfg, args.cpu_seconds)
     if rank == 0:
@@ -432,6 +523,10 @@ def main():
     ap.add_argument("--e2e-runs", type=int, default=20, help="runs (half FIX, half RND) in the host-records e2e leg")
     ap.add_argument("--breakdown", action="store_true", help="host-timed per-call breakdown (syncs between calls)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--scaling", default="auto", choices=["auto", "weak", "strong"],
+                    help="auto: strong for C5 (the scaling sweep: 1000 runs split across the ranks), weak otherwise")
+    ap.add_argument("--hbm-budget-gb", type=float, default=140.0, help="records resident at once per GPU")
+    ap.add_argument("--e2e-gb", type=float, default=8.0, help="pinned host bytes of the e2e leg's runs (bound)")
     args = ap.parse_args()
     import __graft_entry__
     __graft_entry__.build_native()
