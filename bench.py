@@ -23,6 +23,8 @@ import sys
 import threading
 import time
 
+import numpy as np
+
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
@@ -376,6 +378,8 @@ def run_ours(args):
             lk = ctx.leak_test(ef, er, 0.05)
         tick("leak_test", t0)
         out.update(n_diff=len(d), n_leaks=len(lk), info_f=ef.info(), info_r=er.info())
+        if args.dump:
+            out.update(diff_rows=np.array(d), leak_rows=np.array(lk))
 
     def step():
         if resident:
@@ -504,6 +508,12 @@ def run_ours(args):
         res["e2e"] = e2e_leg(args, p, api, tracegen, dev, stream, e2e_runs, my_runs, world, rank)
     if rank == 0 and not args.no_cpu:
         res["cpu_baseline"] = cpu_baseline(cfg, args.cpu_seconds)
+    if rank == 0 and args.dump:  # the last step's result rows (tests: the N > 1 path against the oracle)
+        os.makedirs(args.dump, exist_ok=True)
+        np.save(os.path.join(args.dump, "diff.npy"), out["diff_rows"])
+        np.save(os.path.join(args.dump, "leaks.npy"), out["leak_rows"])
+        with open(os.path.join(args.dump, "runs.json"), "w") as f:
+            json.dump({"config": cfg, "runs_fix": p.runs_fix, "runs_rnd": p.runs_rnd, "runs": all_runs}, f)
     if rank == 0:
         print(json.dumps(res), flush=True)
     if world > 1:
@@ -527,6 +537,7 @@ def main():
                     help="auto: strong for C5 (the scaling sweep: 1000 runs split across the ranks), weak otherwise")
     ap.add_argument("--hbm-budget-gb", type=float, default=140.0, help="records resident at once per GPU")
     ap.add_argument("--e2e-gb", type=float, default=8.0, help="pinned host bytes of the e2e leg's runs (bound)")
+    ap.add_argument("--dump", default="", help="rank 0 writes the last step's diff / leak rows here (tests)")
     args = ap.parse_args()
     import __graft_entry__
     __graft_entry__.build_native()

@@ -46,6 +46,33 @@ __global__ void scatter_owner_kernel(const Key128* k, const unsigned long long* 
   }
 }
 
+/* the same two passes straight over a hash table's buckets (no canonical sort first): empty cells skipped */
+__global__ void count_owner_table_kernel(const owl_bucket* b, uint64_t cap, int tbl, int world,
+                                         unsigned long long* counts) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < cap; i += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long hi = b[i >> 1].key[i & 1][0];
+    if (hi != OWL_EMPTY_KEY) atomicAdd(&counts[owner_of(hi, tbl, world)], 1ull);
+  }
+}
+
+__global__ void scatter_owner_table_kernel(const owl_bucket* b, uint64_t cap, int tbl, int world,
+                                           const unsigned long long* offs, unsigned long long* cursor,
+                                           ExchangeCell* out) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < cap; i += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long hi = b[i >> 1].key[i & 1][0];
+    if (hi == OWL_EMPTY_KEY) continue;
+    const uint32_t o = owner_of(hi, tbl, world);
+    const unsigned long long pos = offs[o] + atomicAdd(&cursor[o], 1ull);
+    ExchangeCell e;
+    e.hi = hi;
+    e.lo = b[i >> 1].key[i & 1][1];
+    e.count = b[i >> 1].count[i & 1];
+    e.tbl = (uint32_t)tbl;
+    e._pad = 0;
+    out[pos] = e;
+  }
+}
+
 __global__ void absorb_kernel(DevTable t0, DevTable t1, DevTable t2, DevTable t3, const ExchangeCell* cells, uint64_t n,
                               FoldStatus* st) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
@@ -90,6 +117,45 @@ cudaError_t owl_partition_cells(const SortedTable* tabs, int world, ExchangeCell
     if (tabs[t].n)
       scatter_owner_kernel<<<grid_for(tabs[t].n, 256), 256, 0, st>>>(tabs[t].k, tabs[t].c, tabs[t].n, t, world, doff,
                                                                      dcur, *d_send);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  owl_dev_free(dcnt); owl_dev_free(doff); owl_dev_free(dcur);
+  return e == cudaSuccess ? cudaGetLastError() : e;
+}
+
+cudaError_t owl_partition_tables(const DevTable* tabs, int world, ExchangeCell** d_send, uint64_t* counts,
+                                 cudaStream_t st) {
+  unsigned long long *dcnt = nullptr, *doff = nullptr, *dcur = nullptr;
+  std::vector<unsigned long long> fill(T_NUM, 0);
+  cudaError_t e = cudaSuccess;
+  for (int t = 0; t < T_NUM && e == cudaSuccess; ++t)
+    if (tabs[t].b) e = cudaMemcpyAsync(&fill[t], tabs[t].fill, 8, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return e;
+  uint64_t total = 0;
+  for (int t = 0; t < T_NUM; ++t) total += fill[t];
+  dcnt = (unsigned long long*)owl_dev_alloc(world * 8);
+  doff = (unsigned long long*)owl_dev_alloc(world * 8);
+  dcur = (unsigned long long*)owl_dev_alloc(world * 8);
+  *d_send = (ExchangeCell*)owl_dev_alloc((total + 1) * sizeof(ExchangeCell));
+  if (!dcnt || !doff || !dcur || !*d_send) {
+    owl_dev_free(dcnt); owl_dev_free(doff); owl_dev_free(dcur); owl_dev_free(*d_send);
+    return cudaErrorMemoryAllocation;
+  }
+  cudaMemsetAsync(dcnt, 0, world * 8, st);
+  cudaMemsetAsync(dcur, 0, world * 8, st);
+  for (int t = 0; t < T_NUM; ++t)
+    if (tabs[t].b && fill[t])
+      count_owner_table_kernel<<<grid_for(tabs[t].cap, 256), 256, 0, st>>>(tabs[t].b, tabs[t].cap, t, world, dcnt);
+  std::vector<unsigned long long> h(world), off(world);
+  e = cudaMemcpyAsync(h.data(), dcnt, world * 8, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  unsigned long long acc = 0;
+  for (int w = 0; w < world; ++w) { off[w] = acc; acc += h[w]; counts[w] = h[w]; }
+  if (e == cudaSuccess) e = cudaMemcpyAsync(doff, off.data(), world * 8, cudaMemcpyHostToDevice, st);
+  for (int t = 0; t < T_NUM && e == cudaSuccess; ++t)
+    if (tabs[t].b && fill[t])
+      scatter_owner_table_kernel<<<grid_for(tabs[t].cap, 256), 256, 0, st>>>(tabs[t].b, tabs[t].cap, t, world, doff,
+                                                                             dcur, *d_send);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   owl_dev_free(dcnt); owl_dev_free(doff); owl_dev_free(dcur);
   return e == cudaSuccess ? cudaGetLastError() : e;

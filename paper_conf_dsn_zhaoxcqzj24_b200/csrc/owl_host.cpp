@@ -1109,11 +1109,17 @@ OWL_API owl_status owl_partition_evidence(owl_ctx* ctx, const owl_adcfg* partial
   if (!ctx || !partial || world < 1 || !d_send || !send_bytes) return fail(OWL_ERR_INVALID_ARG, "bad argument");
   CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
   owl_adcfg* g = const_cast<owl_adcfg*>(partial);
-  owl_status s = ensure_sorted(g);
-  if (s != OWL_OK) return s;
   if (g->send) { owl_dev_free(g->send); g->send = nullptr; }
   std::vector<uint64_t> counts(world);
-  CUDA_TRY(owl_partition_cells(g->sorted, world, &g->send, counts.data(), ctx->stream), "partition");
+  bool tables = true; /* pack straight from the hash tables; an evidence that kept only its sorted cells uses those */
+  for (int t = 0; t < T_NUM; ++t) tables = tables && g->tab[t].b;
+  if (tables) {
+    CUDA_TRY(owl_partition_tables(g->tab, world, &g->send, counts.data(), ctx->stream), "partition");
+  } else {
+    owl_status s = ensure_sorted(g);
+    if (s != OWL_OK) return s;
+    CUDA_TRY(owl_partition_cells(g->sorted, world, &g->send, counts.data(), ctx->stream), "partition");
+  }
   for (int w = 0; w < world; ++w) send_bytes[w] = counts[w] * sizeof(ExchangeCell);
   *d_send = g->send;
   return OWL_OK;

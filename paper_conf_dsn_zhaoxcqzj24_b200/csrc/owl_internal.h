@@ -164,6 +164,9 @@ struct ExchangeCell {
 };
 cudaError_t owl_partition_cells(const SortedTable* tabs, int world, ExchangeCell** d_send, uint64_t* counts,
                                 cudaStream_t st);
+/* the same straight from the (unsorted) hash tables: no canonical sort before the exchange */
+cudaError_t owl_partition_tables(const DevTable* tabs, int world, ExchangeCell** d_send, uint64_t* counts,
+                                 cudaStream_t st);
 cudaError_t owl_absorb_cells(const DevTable* tabs, const ExchangeCell* cells, uint64_t n, FoldStatus* st_dev,
                              cudaStream_t st);
 
