@@ -2,14 +2,16 @@
  * owl_fold.cu — A1-A3: stream trace records once and fold them thread -> warp -> kernel into the
  * A-DCFG hash tables (§V.A-B).
  *
- * Design v12 (every variant and its measurement in profiles/r01_v4_ab.txt): the fold is an
- * HBM stream whose per-record work must fit the issue budget, and at 24 warps per SM the register budget
- * (80) binds, so every choice below minimises instructions per 32-record chunk and live registers:
+ * Design v16 (the variants and their measurements: profiles/r01_v4_ab.txt, and for the round-2
+ * redesign attempts profiles/r02_fold_experiments.txt).  The fold is an HBM stream whose per-record work must
+ * fit the issue budget; at 24 warps per SM the register budget (80) binds, so every choice below minimises
+ * instructions per 32-record chunk and live registers:
  *
  *  * persistent CTAs of FOLD_WARPS independent warps; a warp pops one work item (segment, tile of 2^15
  *    records) at a time from a global counter.  A tile holds the traced warps whose first record lies in
  *    it: the warp finds the first such start with a 33-ary warp-cooperative search and finishes the last
- *    traced warp past the tile end;
+ *    traced warp past the tile end.  Every segment's walked records are counted (= n iff the warp-major
+ *    layout held) and every traced warp start is marked in a bitmap (a warp seen twice is not warp-major);
  *  * a warp walks its traced warp FOLD_U chunks of 32 records at a time (one 128-bit streaming load per
  *    lane and chunk), with cp.async.bulk.prefetch.L2 keeping the next granules of its stream in flight;
  *  * A2: a chunk of 32 well-formed MEM records of the current basic block is the fast path (context
@@ -22,14 +24,17 @@
  *  * A3, "merging identical thread traces" before any global atomic: a broadcast chunk (32
  *    equal keys) is one add of 32; every lane then looks its key up on its own in the CTA directory
  *    (hot broadcast cells hold their count there; a hot 1 KB address window of one attribute owns a page
- *    of keyless 4-byte bins and the lane adds 1 to its bin).  Keys enter the directory on their 16th
- *    sighting (4-way bucketed filter), so one-off windows never take pages.  Lanes that miss insert into
- *    the global open-addressing table: first probes of the step's chunks in flight together, counts added
- *    with fire-and-forget RED.64 in L2.
- *    The shared directory / pages / CF cells are exact partial sums, flushed to the global tables when
- *    the CTA finishes.
+ *    of keyless 4-byte bins and the lane adds 1 to its bin).  Keys enter the directory on their ADMIT-th
+ *    (6th) sighting, counted in a 4-way bucketed filter, so one-off windows never take pages.  Lanes that
+ *    miss insert into the global open-addressing table: first probes of the step's chunks in flight
+ *    together, counts added with fire-and-forget RED.64 in L2.
+ *    The shared directory / pages / CF cells are exact partial sums, flushed to the global tables when the
+ *    CTA finishes.  Directory and page counters close at SHARED_TOTAL_LIMIT walked records per CTA; the CF
+ *    cells' 32-bit counters are bounded by the BB entries a CTA walks in one launch (< 2^32 for any launch
+ *    that fits in device memory: at most 180 GB / 16 B = 1.1e10 records).
  * Malformed records are reported with the minimum (segment, index) and skipped (state unaffected),
- * exactly as the oracle does.
+ * exactly as the oracle does (bucketed channel-order segments are mapped back to the caller's order by
+ * owl_first_bad_record after the fold).
  */
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -125,26 +130,13 @@ struct __align__(16) FoldSmem {
   unsigned int off;          /* 1: shared counting closed (total limit, or experiment mode 8) */
 };
 
-__device__ __forceinline__ uint64_t evict_first_policy() {
-  uint64_t pol;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-  return pol;
-}
-
-/* Streaming record load: L1 bypassed; no L2 eviction hint by default (v16: the evict_first hint cost 1.8%,
-   2388 -> 2430 GB/s, once the bulk prefetch kept the stream ahead; -DSTREAM_L2_EVICT_FIRST restores it). */
-__device__ __forceinline__ uint4 ld_stream(const uint4* p, uint64_t pol) {
+/* Streaming record load: L1 bypassed, no L2 eviction hint (v16: the evict_first hint cost 1.8% once the bulk
+   prefetch kept the stream ahead) */
+__device__ __forceinline__ uint4 ld_stream(const uint4* p, uint64_t) {
   uint4 r;
-#ifndef STREAM_L2_EVICT_FIRST
-  (void)pol;
   asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
                : "l"(p));
-#else
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
-               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
-               : "l"(p), "l"(pol));
-#endif
   return r;
 }
 
@@ -640,11 +632,7 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         shared_on = !*(volatile unsigned int*)&s.off;
       }
       uint4 rr[FOLD_U];
-#ifdef STREAM_L2_EVICT_FIRST
-      const uint64_t pol = evict_first_policy(); /* one instruction: cheaper than a live register pair */
-#else
       const uint64_t pol = 0;
-#endif
       if (w.p + 32 * FOLD_U <= end) {
 #pragma unroll
         for (int u = 0; u < FOLD_U; ++u) rr[u] = ld_stream(w.p + u * 32 + lane, pol);

@@ -20,12 +20,20 @@
 #include <vector>
 
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "owl.h"
 #include "owl_internal.h"
 #include "owl_myers.h"
 
 #define OWL_API extern "C" __attribute__((visibility("default")))
+
+/* NVTX range around an ABI call (visible in nsys / ncu timelines; free when no tool is attached) */
+struct OwlRange {
+  explicit OwlRange(const char* name) { nvtxRangePushA(name); }
+  ~OwlRange() { nvtxRangePop(); }
+};
+#define OWL_RANGE() OwlRange owl_range_(__func__)
 
 namespace {
 
@@ -620,6 +628,7 @@ OWL_API owl_status owl_ctx_set_config(owl_ctx* ctx, const owl_config* cfg) {
 }
 
 OWL_API owl_status owl_ingest_traces(owl_ctx* ctx, const owl_segment* segs, size_t n_segs, owl_stream_t stream) {
+  OWL_RANGE();
   if (!ctx || (!segs && n_segs)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
   for (size_t i = 0; i < n_segs; ++i) {
     const owl_segment& s = segs[i];
@@ -663,6 +672,7 @@ OWL_API owl_status owl_register_remote_runs(owl_ctx* ctx, const uint32_t* runs, 
 }
 
 OWL_API owl_status owl_build_adcfg(owl_ctx* ctx, const uint32_t* runs, size_t n_runs, owl_adcfg** out) {
+  OWL_RANGE();
   if (!ctx || !out || (!runs && n_runs)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
   *out = nullptr;
   CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
@@ -678,6 +688,7 @@ OWL_API owl_status owl_build_adcfg(owl_ctx* ctx, const uint32_t* runs, size_t n_
 }
 
 OWL_API owl_status owl_adcfg_accumulate(owl_ctx* ctx, owl_adcfg* g, const uint32_t* runs, size_t n_runs) {
+  OWL_RANGE();
   if (!ctx || !g || (!runs && n_runs)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
   if (!n_runs) return OWL_OK;
   CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
@@ -722,6 +733,7 @@ OWL_API owl_status owl_adcfg_destroy(owl_adcfg* g) {
 }
 
 OWL_API owl_status owl_adcfg_export(const owl_adcfg* gc, const char* path, void** host_blob, size_t* bytes) {
+  OWL_RANGE();
   if (!gc) return fail(OWL_ERR_INVALID_ARG, "NULL adcfg");
   owl_adcfg* g = const_cast<owl_adcfg*>(gc);
   CUDA_TRY(cudaSetDevice(g->ctx->device), "cudaSetDevice");
@@ -777,6 +789,7 @@ OWL_API owl_status owl_adcfg_export(const owl_adcfg* gc, const char* path, void*
 }
 
 OWL_API owl_status owl_diff_adcfg(owl_ctx* ctx, const owl_adcfg* a, const owl_adcfg* b, owl_diff** rows, size_t* n_rows) {
+  OWL_RANGE();
   if (!ctx || !a || !b || !rows || !n_rows) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
   CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
   owl_adcfg* ga = const_cast<owl_adcfg*>(a);
@@ -890,6 +903,7 @@ owl_status run_ks(owl_ctx* ctx, const owl_adcfg* f, const owl_adcfg* r, double s
 
 OWL_API owl_status owl_ks_tests(owl_ctx* ctx, const owl_adcfg* e_fix, const owl_adcfg* e_rnd, double significance,
                                 owl_ks_row** rows, size_t* n_rows) {
+  OWL_RANGE();
   if (!ctx || !e_fix || !e_rnd || !rows || !n_rows) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
   CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
   Alignment al = align(e_fix, e_rnd);
@@ -906,6 +920,7 @@ OWL_API owl_status owl_ks_tests(owl_ctx* ctx, const owl_adcfg* e_fix, const owl_
    comparisons with each class's representative decide. */
 OWL_API owl_status owl_filter_inputs(owl_ctx* ctx, const uint32_t* runs, size_t n_runs, uint32_t* class_of,
                                      uint32_t* n_classes) {
+  OWL_RANGE();
   if (!ctx || !n_classes || (n_runs && (!runs || !class_of))) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
   for (size_t i = 0; i < n_runs; ++i)
     for (size_t j = 0; j < i; ++j)
@@ -1015,6 +1030,7 @@ void order_ks_leaks(const Alignment& al, std::vector<owl_leak>& rows, std::vecto
 
 OWL_API owl_status owl_leak_test(owl_ctx* ctx, const owl_adcfg* f, const owl_adcfg* r, double significance,
                                  owl_leak** leaks, size_t* n_leaks) {
+  OWL_RANGE();
   if (!ctx || !f || !r || !leaks || !n_leaks) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
   CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
   const uint32_t NA = 0xFFFFFFFFu;
@@ -1047,6 +1063,7 @@ OWL_API owl_status owl_leak_test(owl_ctx* ctx, const owl_adcfg* f, const owl_adc
 
 OWL_API owl_status owl_merge_leaks(owl_ctx* ctx, const owl_adcfg* f, const owl_adcfg* r, const owl_leak* parts,
                                    size_t n_parts, owl_leak** leaks, size_t* n_leaks) {
+  OWL_RANGE();
   if (!ctx || !f || !r || !leaks || !n_leaks || (n_parts && !parts)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
   Alignment al = align(f, r);
   std::vector<owl_leak> out, ks;
@@ -1067,6 +1084,7 @@ OWL_API owl_status owl_merge_leaks(owl_ctx* ctx, const owl_adcfg* f, const owl_a
 
 OWL_API owl_status owl_merge_diffs(owl_ctx* ctx, const owl_adcfg* a, const owl_adcfg* b, const owl_diff* parts,
                                    size_t n_parts, owl_diff** rows, size_t* n_rows) {
+  OWL_RANGE();
   if (!ctx || !a || !b || !rows || !n_rows || (n_parts && !parts)) return fail(OWL_ERR_INVALID_ARG, "NULL argument");
   std::vector<owl_diff> out;
   for (size_t i = 0; i < n_parts; ++i) {
@@ -1106,6 +1124,7 @@ OWL_API owl_status owl_merge_diffs(owl_ctx* ctx, const owl_adcfg* a, const owl_a
 
 OWL_API owl_status owl_partition_evidence(owl_ctx* ctx, const owl_adcfg* partial, int world, void** d_send,
                                           uint64_t* send_bytes) {
+  OWL_RANGE();
   if (!ctx || !partial || world < 1 || !d_send || !send_bytes) return fail(OWL_ERR_INVALID_ARG, "bad argument");
   CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");
   owl_adcfg* g = const_cast<owl_adcfg*>(partial);
@@ -1127,6 +1146,7 @@ OWL_API owl_status owl_partition_evidence(owl_ctx* ctx, const owl_adcfg* partial
 
 OWL_API owl_status owl_absorb_evidence(owl_ctx* ctx, const owl_adcfg* like, const void* d_recv, const uint64_t* recv_bytes,
                                        int world, int rank, owl_adcfg** owned) {
+  OWL_RANGE();
   (void)rank;
   if (!ctx || !like || world < 1 || !owned || !recv_bytes) return fail(OWL_ERR_INVALID_ARG, "bad argument");
   CUDA_TRY(cudaSetDevice(ctx->device), "cudaSetDevice");

@@ -125,13 +125,6 @@ void owl_sorted_free(SortedTable* s);
 cudaError_t owl_table_insert_sorted(const DevTable& t, int tbl, const Key128* k, const unsigned long long* c,
                                     uint64_t n, FoldStatus* st_dev, cudaStream_t st);
 
-struct DiffCell {
-  Key128 k;
-  unsigned long long ca, cb;
-};
-/* full outer join of two sorted tables: the differing cells in canonical order */
-cudaError_t owl_diff_sorted(const SortedTable& a, const SortedTable& b, std::vector<DiffCell>& out, cudaStream_t st);
-
 /* A5 over all tables at once (canonical order), into malloc'd host rows with room for extra_rows more */
 cudaError_t owl_diff_rows(const SortedTable* A, const SortedTable* B, int ntab, owl_diff** rows, uint64_t* n_rows,
                           size_t extra_rows, cudaStream_t st);

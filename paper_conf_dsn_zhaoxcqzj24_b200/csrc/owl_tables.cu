@@ -144,20 +144,6 @@ __global__ void diff_flag_kernel(const Key128* ak, const unsigned long long* ac,
     fb[i] = find_key(ak, na, bk[i]) >= na ? 1 : 0;
 }
 
-__global__ void gather_diff_kernel(const uint64_t* idx, const unsigned long long* nsel, const Key128* k,
-                                   const unsigned long long* c, const unsigned long long* other, int a_side,
-                                   DiffCell* out) {
-  const uint64_t n = *nsel;
-  for (uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; t < n; t += (uint64_t)gridDim.x * blockDim.x) {
-    const uint64_t i = idx[t];
-    DiffCell d;
-    d.k = k[i];
-    if (a_side) { d.ca = c[i]; d.cb = other[i]; }
-    else { d.ca = 0; d.cb = c[i]; }
-    out[t] = d;
-  }
-}
-
 /* key = gwarp, with every out-of-range gwarp mapped to n_warps (a stable sort keeps their relative order;
    the fold reports the first of them): the sort needs only ceil(log2(n_warps + 1)) bits */
 __global__ void bucket_keys_kernel(const uint4* rec, uint64_t n, uint32_t n_warps, uint32_t* gw, uint64_t* idx) {
@@ -371,64 +357,6 @@ cudaError_t owl_table_insert_sorted(const DevTable& t, int tbl, const Key128* k,
   if (!n) return cudaSuccess;
   insert_sorted_kernel<<<grid_for(n, 256), 256, 0, st>>>(t, tbl, k, c, n, st_dev);
   return cudaGetLastError();
-}
-
-cudaError_t owl_diff_sorted(const SortedTable& a, const SortedTable& b, std::vector<DiffCell>& out, cudaStream_t st) {
-  out.clear();
-  const uint64_t na = a.n, nb = b.n;
-  unsigned char* fa = (unsigned char*)owl_dev_alloc(na + 1);
-  unsigned char* fb = (unsigned char*)owl_dev_alloc(nb + 1);
-  unsigned long long* cboa = (unsigned long long*)owl_dev_alloc((na + 1) * 8);
-  uint64_t* ia = (uint64_t*)owl_dev_alloc((na + 1) * 8);
-  uint64_t* ib = (uint64_t*)owl_dev_alloc((nb + 1) * 8);
-  unsigned long long* nsel = (unsigned long long*)owl_dev_alloc(16);
-  DiffCell* da = (DiffCell*)owl_dev_alloc((na + 1) * sizeof(DiffCell));
-  DiffCell* db = (DiffCell*)owl_dev_alloc((nb + 1) * sizeof(DiffCell));
-  cudaError_t e = cudaSuccess;
-  void* dt = nullptr;
-  if (!fa || !fb || !cboa || !ia || !ib || !nsel || !da || !db) e = cudaErrorMemoryAllocation;
-  if (e == cudaSuccess) {
-    diff_flag_kernel<<<grid_for(na > nb ? na : nb, 256), 256, 0, st>>>(a.k, a.c, na, b.k, b.c, nb, fa, cboa, fb);
-    size_t tmp = 0, tmp2 = 0;
-    cub::DeviceSelect::Flagged(nullptr, tmp, thrust::counting_iterator<uint64_t>(0), fa, ia, nsel, (int64_t)na, st);
-    cub::DeviceSelect::Flagged(nullptr, tmp2, thrust::counting_iterator<uint64_t>(0), fb, ib, nsel + 1, (int64_t)nb, st);
-    if (tmp2 > tmp) tmp = tmp2;
-    dt = owl_dev_alloc(tmp);
-    if (!dt) e = cudaErrorMemoryAllocation;
-  }
-  unsigned long long hn[2] = {0, 0};
-  if (e == cudaSuccess) {
-    size_t tmp = 0;
-    cub::DeviceSelect::Flagged(nullptr, tmp, thrust::counting_iterator<uint64_t>(0), fa, ia, nsel, (int64_t)na, st);
-    e = cub::DeviceSelect::Flagged(dt, tmp, thrust::counting_iterator<uint64_t>(0), fa, ia, nsel, (int64_t)na, st);
-    tmp = 0;
-    cub::DeviceSelect::Flagged(nullptr, tmp, thrust::counting_iterator<uint64_t>(0), fb, ib, nsel + 1, (int64_t)nb, st);
-    if (e == cudaSuccess)
-      e = cub::DeviceSelect::Flagged(dt, tmp, thrust::counting_iterator<uint64_t>(0), fb, ib, nsel + 1, (int64_t)nb, st);
-    if (e == cudaSuccess) {
-      gather_diff_kernel<<<grid_for(na, 256), 256, 0, st>>>(ia, nsel, a.k, a.c, cboa, 1, da);
-      gather_diff_kernel<<<grid_for(nb, 256), 256, 0, st>>>(ib, nsel + 1, b.k, b.c, nullptr, 0, db);
-      e = cudaMemcpyAsync(hn, nsel, 16, cudaMemcpyDeviceToHost, st);
-    }
-    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  }
-  std::vector<DiffCell> ha(hn[0]), hb(hn[1]);
-  if (e == cudaSuccess && hn[0]) e = cudaMemcpy(ha.data(), da, hn[0] * sizeof(DiffCell), cudaMemcpyDeviceToHost);
-  if (e == cudaSuccess && hn[1]) e = cudaMemcpy(hb.data(), db, hn[1] * sizeof(DiffCell), cudaMemcpyDeviceToHost);
-  if (e == cudaSuccess) { /* merge the two canonical-order lists */
-    out.reserve(ha.size() + hb.size());
-    size_t i = 0, j = 0;
-    while (i < ha.size() || j < hb.size()) {
-      if (j >= hb.size() || (i < ha.size() && (ha[i].k.hi < hb[j].k.hi ||
-                                                (ha[i].k.hi == hb[j].k.hi && ha[i].k.lo < hb[j].k.lo))))
-        out.push_back(ha[i++]);
-      else
-        out.push_back(hb[j++]);
-    }
-  }
-  owl_dev_free(fa); owl_dev_free(fb); owl_dev_free(cboa); owl_dev_free(ia); owl_dev_free(ib);
-  owl_dev_free(nsel); owl_dev_free(da); owl_dev_free(db); owl_dev_free(dt);
-  return e;
 }
 
 namespace {

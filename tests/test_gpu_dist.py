@@ -34,7 +34,7 @@ def _port():
     return p
 
 
-@pytest.mark.parametrize("cfg,runs", [(9, 6), (4, 2)])
+@pytest.mark.parametrize("cfg,runs", [(9, 6), (2, 2)])
 def test_bench_two_ranks_equal_oracle(tmp_path, cfg, runs):
     env = dict(os.environ, OWL_BENCH_SHARE_GPU="1")
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
