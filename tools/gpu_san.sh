@@ -1,3 +1,10 @@
+#!/bin/bash
+# compute-sanitizer memcheck / racecheck / synccheck over tools/san_case.py (C1 full, C2 slices, config 9);
+# summaries to gpurun_out/san_<tool>.txt
 mkdir -p gpurun_out
-timeout 600 compute-sanitizer --tool memcheck --show-backtrace device python -m pytest tests -m gpu -q -x -k "config_parity and 2-32" > gpurun_out/san.txt 2>&1
-grep -m 20 -E "=========|Invalid|Illegal|at 0x|owl_fold" gpurun_out/san.txt | head -40
+for tool in memcheck racecheck synccheck; do
+  extra=""
+  [ $tool = racecheck ] && extra="--racecheck-report hazard"
+  timeout 1500 compute-sanitizer --tool $tool $extra --print-limit 200 python tools/san_case.py > gpurun_out/san_$tool.txt 2>&1
+  echo "== $tool rc=$?"; grep -E "ERROR SUMMARY|RACECHECK SUMMARY|hazard|C[0-9] div" gpurun_out/san_$tool.txt | sort | uniq -c | head -20
+done
