@@ -206,12 +206,14 @@ def e2e_leg(args, p, api, tracegen, dev, stream, n_runs_e2e, my_runs, world=1, r
     for r in runs_f + runs_r:
         for m in tracegen.run_segments(p, r):
             buf, n = tracegen.device_records(p, r, m.seq, device=dev, stream=stream)
+            if args.channel_order:
+                buf = tracegen.device_interleave(buf, n)
             h = torch.empty(buf.shape, dtype=buf.dtype, pin_memory=True)
             h.copy_(buf)
             del buf
             hold.append(h)
             segs.append(api.Segment(base_run + r, m.input_class, m.seq, m.n_warps, m.kernel_id, h, n,
-                                    flags=api.OWL_SEG_WARP_MAJOR | api.OWL_SEG_HOST_RECORDS))
+                                    flags=api.OWL_SEG_HOST_RECORDS | (0 if args.channel_order else api.OWL_SEG_WARP_MAJOR)))
             n_rec += n
     torch.cuda.synchronize()
     ctx.ingest(segs, stream)
@@ -327,7 +329,10 @@ def run_ours(args):
         for r in runs:
             for m in tracegen.run_segments(p, r):
                 buf, n = tracegen.device_records(p, r, m.seq, device=dev, stream=stream)
-                segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, n))
+                if args.channel_order:  # a tracer channel's order (reading R17): bursts of 32, warps round-robin
+                    buf = tracegen.device_interleave(buf, n)
+                segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, n,
+                                        flags=0 if args.channel_order else api.OWL_SEG_WARP_MAJOR))
         torch.cuda.synchronize()
         return segs
 
@@ -473,7 +478,9 @@ def run_ours(args):
         "metric": METRIC, "value": value, "unit": "records/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": mode,
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-        "config": {"workload": tracegen.CONFIG_NAMES[cfg], "runs_per_gpu": len(my_runs), "runs_total": p.n_runs,
+        "config": {"workload": tracegen.CONFIG_NAMES[cfg] + (" (channel order)" if args.channel_order else ""),
+                   "record_order": "channel (bursts of 32, warps round-robin)" if args.channel_order else "warp-major",
+                   "runs_per_gpu": len(my_runs), "runs_total": p.n_runs,
                    "records_per_gpu": n_records, "bytes_per_gpu": 16 * n_records,
                    "l2": "inputs (%.1f GB) >> 126 MB L2; no flush needed" % (16 * n_records / 1e9),
                    "parallelism": f"dp{world} (runs sharded, key-hash exchange, {mode} scaling)" if world > 1
@@ -537,6 +544,8 @@ def main():
                     help="auto: strong for C5 (the scaling sweep: 1000 runs split across the ranks), weak otherwise")
     ap.add_argument("--hbm-budget-gb", type=float, default=140.0, help="records resident at once per GPU")
     ap.add_argument("--e2e-gb", type=float, default=8.0, help="pinned host bytes of the e2e leg's runs (bound)")
+    ap.add_argument("--channel-order", action="store_true",
+                    help="records in a tracer channel's order (bursts of 32 per warp, warps round-robin; N2)")
     ap.add_argument("--dump", default="", help="rank 0 writes the last step's diff / leak rows here (tests)")
     args = ap.parse_args()
     import __graft_entry__

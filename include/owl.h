@@ -69,14 +69,16 @@ enum { OWL_FIXED = 0, OWL_RANDOM = 1 }; /* input classes of the leakage-analysis
 
 enum {
   /* Records of each traced warp are contiguous in the buffer (any warp order).  Without this flag only
-     per-warp program order is guaranteed (reading R17) and the library first buckets the records by
-     gwarp, stably, into a scratch buffer (3x the record bytes). */
+     per-warp program order is guaranteed (reading R17, a tracer channel's order) and the build first buckets
+     the records by gwarp on the device: the runs of consecutive records of one warp ("bursts") are found in
+     one streaming pass, the bursts (not the records) are sorted stably by warp and copied whole into a
+     warp-major scratch buffer (the segment's bytes again, plus 9 B per burst). */
   OWL_SEG_WARP_MAJOR = 1u,
   /* `records` is a HOST pointer (pinned for asynchronous copies; pageable works but copies synchronously).
      owl_build_adcfg stages host segments in waves of at most owl_config.host_chunk_bytes (a wave holds at
      least one whole segment) through two device buffers: the copy of the next wave overlaps the fold of the
      current one, so device memory for host records stays at 2 x the largest wave.  A channel-order host
-     segment is additionally bucketed by warp (3x its bytes of scratch until the build returns). */
+     segment is additionally bucketed by warp (its bytes again of scratch until the build returns). */
   OWL_SEG_HOST_RECORDS = 2u
 };
 

@@ -226,8 +226,9 @@ const char* kerr_text(uint32_t code) {
    Device-resident segments are folded in one launch.  Host segments (OWL_SEG_HOST_RECORDS) are staged in waves
    of at most host_chunk_bytes (a wave holds at least one segment) through two device buffers: the copy of wave
    k + 1 (copy stream) overlaps the fold of wave k (context stream), and a buffer is refilled only after the fold
-   that read it.  Channel-order segments are bucketed by warp on the device first (3x their bytes of scratch,
-   held until the pass returns: the error report of a malformed record maps it back through the permutation). */
+   that read it.  The channel-order segments of each launch are bucketed by warp on the device first, together
+   and by bursts (their bytes again + 9 B per burst of scratch, held until the pass returns: the error report of
+   a malformed record maps it back to the caller's order through its burst). */
 owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable* tab, unsigned* overflow,
                      uint64_t* n_records) {
   const cudaStream_t st = ctx->stream;
@@ -235,7 +236,8 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
   const uint32_t tile_shift = getenv("OWL_TILE_SHIFT") ? (uint32_t)atoi(getenv("OWL_TILE_SHIFT")) : 15u; /* tile sweep: profiles/r01_v4_ab.txt */
   std::vector<FoldSeg> fs(plan.size());
   std::vector<void*> scratch;
-  std::vector<uint64_t*> perms(plan.size(), nullptr);
+  std::vector<BucketedSet> sets; /* channel-order segments, bucketed per launch */
+  std::vector<std::pair<uint32_t, uint32_t>> bucketed(plan.size(), {~0u, 0u}); /* (set, position) */
   uint64_t seen_words = 0, nrec = 0;
   for (size_t i = 0; i < plan.size(); ++i) seen_words += (plan[i].s.n_warps + 31) / 32;
   uint32_t* seen = (uint32_t*)owl_dev_alloc((seen_words + 1) * 4);
@@ -334,21 +336,29 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
       if (e != cudaSuccess) { status = cuda_fail(e, "fold: H2D staging"); break; }
     }
     if (w >= 1) cudaStreamWaitEvent(st, ready[(w - 1) & 1], 0);
-    /* channel order: stable bucket by warp (R17) */
-    for (size_t i : launches[w]) {
-      const owl_segment& s = plan[i].s;
-      if (!s.n_records || (s.flags & OWL_SEG_WARP_MAJOR)) continue;
-      uint4* d = (uint4*)owl_dev_alloc(s.n_records * 16);
-      uint64_t* perm = (uint64_t*)owl_dev_alloc(s.n_records * 8);
-      if (!d || !perm) { owl_dev_free(d); owl_dev_free(perm); status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: bucketing"); break; }
-      scratch.push_back(d);
-      scratch.push_back(perm);
-      cudaError_t e = owl_bucket_by_warp(fs[i].rec, s.n_records, s.n_warps, d, perm, st);
-      if (e != cudaSuccess) { status = cuda_fail(e, "fold: bucketing"); break; }
-      fs[i].rec = d;
-      perms[i] = perm;
+    { /* channel order: the launch's segments bucketed by warp together, by bursts (R17, N2) */
+      std::vector<const uint4*> brec;
+      std::vector<uint64_t> bn;
+      std::vector<uint32_t> bw;
+      std::vector<size_t> bi;
+      for (size_t i : launches[w]) {
+        const owl_segment& s = plan[i].s;
+        if (!s.n_records || (s.flags & OWL_SEG_WARP_MAJOR)) continue;
+        brec.push_back(fs[i].rec);
+        bn.push_back(s.n_records);
+        bw.push_back(s.n_warps);
+        bi.push_back(i);
+      }
+      if (!bi.empty()) {
+        sets.emplace_back();
+        const cudaError_t e = owl_bucket_segments(brec, bn, bw, &sets.back(), st);
+        if (e != cudaSuccess) { status = cuda_fail(e, "fold: bucketing"); break; }
+        for (size_t k = 0; k < bi.size(); ++k) {
+          fs[bi[k]].rec = sets.back().out + sets.back().off[k];
+          bucketed[bi[k]] = {(uint32_t)sets.size() - 1, (uint32_t)k};
+        }
+      }
     }
-    if (status != OWL_OK) break;
     /* work items: (segment, tile of 2^tile_shift records), one range per segment */
     std::vector<FoldSeg> lsegs;
     std::vector<FoldGroup> groups;
@@ -455,9 +465,9 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
       const uint32_t si = (uint32_t)(hs.first_error >> 40);
       uint64_t idx = (hs.first_error >> 3) & ((1ull << 37) - 1);
       uint32_t code = (uint32_t)(hs.first_error & 7);
-      if (si < plan.size() && perms[si]) { /* bucketed: the first bad record in the caller's order */
+      if (si < plan.size() && bucketed[si].first != ~0u) { /* bucketed: the first bad record in the caller's order */
         unsigned long long ic = ~0ull;
-        const cudaError_t e = owl_first_bad_record(fs[si].rec, perms[si], plan[si].s.n_records, plan[si].s.n_warps,
+        const cudaError_t e = owl_first_bad_record(sets[bucketed[si].first], bucketed[si].second, plan[si].s.n_warps,
                                                    &ic, st);
         if (e == cudaSuccess && ic != ~0ull) {
           idx = ic >> 3;
@@ -475,6 +485,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     *overflow = hs.overflow;
   }
   for (void* p : scratch) owl_dev_free(p);
+  for (BucketedSet& b : sets) owl_bucketed_free(&b);
   *n_records = nrec;
   return status;
 }

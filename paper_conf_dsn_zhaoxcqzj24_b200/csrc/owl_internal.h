@@ -132,13 +132,22 @@ cudaError_t owl_diff_rows(const SortedTable* A, const SortedTable* B, int ntab, 
 /* order-independent 128-bit fingerprint of the cells of ntab sorted tables (input-class filtering, N1) */
 cudaError_t owl_tables_fingerprint(const SortedTable* tabs, int ntab, unsigned long long fp[2], cudaStream_t st);
 
-/* the first malformed record (caller's index << 3 | KERR code, ~0 if none) of a bucketed segment */
-cudaError_t owl_first_bad_record(const uint4* rec, const uint64_t* perm, uint64_t n, uint32_t n_warps,
-                                 unsigned long long* idx_code, cudaStream_t st);
-
-/* stable bucketing of a segment's records by gwarp (channel-order input, reading R17) */
-cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, uint4* out, uint64_t* perm,
-                               cudaStream_t st);
+/* Channel-order segments of one fold launch, bucketed by warp together (reading R17, N2): segment s's records in
+   warp-major order at out + off[s]; per sorted burst, its source start (global index in the concatenation of the
+   callers' segments) and its destination start in out. */
+struct BucketedSet {
+  uint4* out = nullptr;
+  uint64_t* bsrc = nullptr;
+  uint64_t* bdst = nullptr;
+  uint64_t nb = 0;
+  std::vector<uint64_t> off;
+};
+cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std::vector<uint64_t>& n,
+                                const std::vector<uint32_t>& n_warps, BucketedSet* out, cudaStream_t st);
+void owl_bucketed_free(BucketedSet* b);
+/* the first malformed record (caller's index in segment seg << 3 | KERR code, ~0 if none) of a bucketed set */
+cudaError_t owl_first_bad_record(const BucketedSet& b, uint32_t seg, uint32_t n_warps, unsigned long long* idx_code,
+                                 cudaStream_t st);
 
 /* KS tests over one table kind (T_TRIPLE: H_cf per node; T_ADDR: H_addr per (bb, ins, j)) */
 struct KsOutRow {

@@ -144,21 +144,6 @@ __global__ void diff_flag_kernel(const Key128* ak, const unsigned long long* ac,
     fb[i] = find_key(ak, na, bk[i]) >= na ? 1 : 0;
 }
 
-/* key = gwarp, with every out-of-range gwarp mapped to n_warps (a stable sort keeps their relative order;
-   the fold reports the first of them): the sort needs only ceil(log2(n_warps + 1)) bits */
-__global__ void bucket_keys_kernel(const uint4* rec, uint64_t n, uint32_t n_warps, uint32_t* gw, uint64_t* idx) {
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t g = rec[i].z;
-    gw[i] = g < n_warps ? g : n_warps;
-    idx[i] = i;
-  }
-}
-
-__global__ void gather_records_kernel(const uint4* rec, const uint64_t* perm, uint64_t n, uint4* out) {
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
-    out[i] = rec[perm[i]];
-}
-
 int grid_for(uint64_t n, int block) {
   uint64_t g = (n + block - 1) / block;
   if (g > 148ull * 16) g = 148ull * 16;
@@ -544,16 +529,160 @@ cudaError_t owl_tables_fingerprint(const SortedTable* tabs, int ntab, unsigned l
 }
 
 namespace {
-/* Error report of a bucketed (channel-order) segment: every malformed record, by the rules of the warp walk
-   (SURVEY §8(b) conventions; the fold's slow path), mapped back to the caller's index; the minimum wins.  One
+/* Channel-order bucketing by bursts (N2).  A tracer's channel delivers each warp's records in runs ("bursts") of
+   consecutive records of one warp.  All channel-order segments of a fold launch are bucketed together and by
+   bursts, not records: one streaming pass marks burst heads (key = (segment, gwarp clamped to n_warps): out-of-
+   range gwarps share one key and keep their stream order), the heads are compacted, the burst keys radix-sorted
+   stably, and every burst is copied whole (coalesced) to its warp-major position in one buffer holding the
+   segments back to back.  Per sorted burst the source start is kept, so a malformed record can be mapped back
+   to the caller's index (owl_first_bad_record) without a per-record permutation. */
+struct BucketArgs {
+  const uint4* const* rec; /* per segment */
+  const uint64_t* off;     /* per segment: first global record index; off[n_seg] = total */
+  const uint32_t* n_warps; /* per segment */
+  uint32_t n_seg;
+  uint32_t warp_bits;      /* key bits of the clamped gwarp */
+};
+
+__device__ __forceinline__ uint32_t seg_of(const BucketArgs& a, uint64_t g) {
+  uint32_t lo = 0, hi = a.n_seg; /* last segment with off <= g */
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (a.off[mid] <= g) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+/* burst heads of one segment, found and compacted in one streaming pass: each warp scans a tile of 1024 records
+   (32 coalesced loads of the gwarp words), keeps its heads in stream order in the tile's slot range of `slots`
+   and the count in tile_cnt; the tiles are concatenated afterwards (burst_gather_kernel) */
+#define BT_LOG 10
+__global__ void burst_head_kernel(const uint4* rec, uint64_t n, uint32_t n_warps, uint64_t goff, uint64_t tile0,
+                                  uint64_t* slots, uint32_t* tile_cnt) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t ntile = (n + (1u << BT_LOG) - 1) >> BT_LOG;
+  const uint64_t wid = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t t = wid; t < ntile; t += nw) {
+    const uint64_t b = t << BT_LOG;
+    uint32_t prev = b == 0 ? 0xFFFFFFFFu : min(__ldg(&rec[b - 1].z), n_warps);
+    uint32_t cnt = 0;
+    uint64_t* out = slots + ((tile0 + t) << BT_LOG);
+    for (int it0 = 0; it0 < (1 << BT_LOG) / 32; it0 += 8) {
+      uint32_t gg[8]; /* 8 loads in flight per lane */
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint64_t i = b + (it0 + u) * 32 + lane;
+        gg[u] = i < n ? __ldg(&rec[i].z) : 0xFFFFFFFEu;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint64_t i = b + (it0 + u) * 32 + lane;
+        const uint32_t g = i < n ? min(gg[u], n_warps) : 0xFFFFFFFEu;
+        uint32_t left = __shfl_up_sync(0xFFFFFFFFu, g, 1);
+        if (lane == 0) left = prev;
+        const bool head = i < n && (i == 0 || g != left);
+        const unsigned m = __ballot_sync(0xFFFFFFFFu, head);
+        if (head) out[cnt + __popc(m & ((1u << lane) - 1))] = goff + i;
+        cnt += __popc(m);
+        prev = __shfl_sync(0xFFFFFFFFu, g, 31);
+      }
+    }
+    if (lane == 0) tile_cnt[tile0 + t] = cnt;
+  }
+}
+
+/* concatenation of the tiles' heads (tile_off = exclusive scan of tile_cnt): global burst starts in stream order */
+__global__ void burst_gather_kernel(const uint64_t* slots, const uint32_t* tile_cnt, const uint64_t* tile_off,
+                                    uint64_t ntile, uint64_t* start) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t wid = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t t = wid; t < ntile; t += nw) {
+    const uint32_t c = tile_cnt[t];
+    for (uint32_t k = lane; k < c; k += 32) start[tile_off[t] + k] = slots[(t << BT_LOG) + k];
+  }
+}
+
+__global__ void widen_kernel(const uint32_t* in, uint64_t n, uint64_t* out) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) out[i] = in[i];
+}
+
+__global__ void burst_key_kernel(const BucketArgs a, const uint64_t* start, const unsigned long long* nb_p,
+                                 unsigned long long* key, uint32_t* id, uint64_t* len, const uint4** ptr) {
+  const uint64_t nb = *nb_p, total = a.off[a.n_seg];
+  for (uint64_t b = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; b < nb; b += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t g = start[b];
+    const uint32_t sg = seg_of(a, g);
+    const uint4* src = a.rec[sg] + (g - a.off[sg]);
+    key[b] = ((unsigned long long)sg << a.warp_bits) | min(src->z, a.n_warps[sg]);
+    id[b] = (uint32_t)b;
+    len[b] = (b + 1 < nb ? start[b + 1] : total) - g; /* a segment's first record is a head: bursts never span */
+    ptr[b] = src;
+  }
+}
+
+__global__ void burst_sorted_kernel(const uint32_t* sid, const uint64_t* start, const uint64_t* len,
+                                    const uint4* const* ptr, const unsigned long long* nb_p, uint64_t* slen,
+                                    uint64_t* bsrc, const uint4** sptr) {
+  const uint64_t nb = *nb_p;
+  for (uint64_t b = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; b < nb; b += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t i = sid[b];
+    slen[b] = len[i];
+    bsrc[b] = start[i];
+    sptr[b] = ptr[i];
+  }
+}
+
+/* sorted bursts copied to their warp-major offsets: each warp takes 4 bursts per round and issues all their
+   loads before the stores (memory-level parallelism); lane k of a burst copies its records k, k + 32, ... */
+__global__ void burst_copy_kernel(const uint4* const* sptr, const uint64_t* slen, const uint64_t* bdst,
+                                  const unsigned long long* nb_p, uint4* out) {
+  const uint64_t nb = *nb_p;
+  const int lane = threadIdx.x & 31;
+  const uint64_t wid = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t b0 = wid * 4; b0 < nb; b0 += nw * 4) {
+    const uint4* src[4];
+    uint64_t l[4], d[4];
+    uint4 v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint64_t b = b0 + u;
+      l[u] = b < nb ? slen[b] : 0;
+      d[u] = b < nb ? bdst[b] : 0;
+      src[u] = b < nb ? sptr[b] : nullptr;
+      if (lane < l[u]) v[u] = src[u][lane];
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (lane < l[u]) out[d[u] + lane] = v[u];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      for (uint64_t k = lane + 32; k < l[u]; k += 32) out[d[u] + k] = src[u][k]; /* bursts longer than 32 */
+  }
+}
+
+/* Error report of a bucketed segment: every malformed record, by the rules of the warp walk (SURVEY §8(b)
+   conventions; the fold's slow path), mapped back to the caller's index through its burst; the minimum wins.  One
    thread per traced warp (start detected on the gwarp change), walking it in order; records with gwarp >=
    n_warps are checked one by one.  Only launched after a fold reported an error in such a segment. */
-__global__ void first_bad_kernel(const uint4* rec, const uint64_t* perm, uint64_t n, uint32_t n_warps,
-                                 unsigned long long* out) {
+__device__ __forceinline__ uint64_t caller_index(uint64_t d, const uint64_t* bsrc, const uint64_t* bdst, uint64_t nb,
+                                                 uint64_t seg_off) {
+  uint64_t lo = 0, hi = nb; /* last burst with bdst <= d */
+  while (hi - lo > 1) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (bdst[mid] <= d) lo = mid; else hi = mid;
+  }
+  return bsrc[lo] + (d - bdst[lo]) - seg_off;
+}
+
+__global__ void first_bad_kernel(const uint4* rec, uint64_t n, uint32_t n_warps, const uint64_t* bsrc,
+                                 const uint64_t* bdst, uint64_t nb, uint64_t seg_off, unsigned long long* out) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t g = rec[i].z;
     if (g >= n_warps) {
-      atomicMin(out, ((unsigned long long)perm[i] << 3) | KERR_GWARP);
+      atomicMin(out, ((unsigned long long)caller_index(seg_off + i, bsrc, bdst, nb, seg_off) << 3) | KERR_GWARP);
       continue;
     }
     if (i > 0 && rec[i - 1].z == g) continue;
@@ -568,44 +697,129 @@ __global__ void first_bad_kernel(const uint4* rec, const uint64_t* perm, uint64_
       } else if ((r.y >> 28) > 8) code = KERR_MTYPE;
       else if (cur == OWL_NONE_BB) code = KERR_NOBB;
       else if (bb != cur) code = KERR_BBMISMATCH;
-      if (code) atomicMin(out, ((unsigned long long)perm[k] << 3) | code);
+      if (code) atomicMin(out, ((unsigned long long)caller_index(seg_off + k, bsrc, bdst, nb, seg_off) << 3) | code);
     }
   }
 }
 }  // namespace
 
-cudaError_t owl_first_bad_record(const uint4* rec, const uint64_t* perm, uint64_t n, uint32_t n_warps,
-                                 unsigned long long* idx_code, cudaStream_t st) {
+void owl_bucketed_free(BucketedSet* b) {
+  owl_dev_free(b->out);
+  owl_dev_free(b->bsrc);
+  owl_dev_free(b->bdst);
+  *b = BucketedSet{};
+}
+
+cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std::vector<uint64_t>& n,
+                                const std::vector<uint32_t>& n_warps, BucketedSet* out, cudaStream_t st) {
+  *out = BucketedSet{};
+  const uint32_t ns = (uint32_t)rec.size();
+  std::vector<uint64_t> off(ns + 1, 0);
+  uint32_t maxw = 1;
+  for (uint32_t i = 0; i < ns; ++i) {
+    off[i + 1] = off[i] + n[i];
+    maxw = std::max(maxw, n_warps[i]);
+  }
+  const uint64_t total = off[ns];
+  out->off = off;
+  if (!total) return cudaSuccess;
+  std::vector<void*> scratch;
+  auto alloc = [&](size_t bytes) { void* p = owl_dev_alloc(bytes); scratch.push_back(p); return p; };
+  uint32_t warp_bits = 1;
+  while (warp_bits < 32 && (1ull << warp_bits) <= (uint64_t)maxw) ++warp_bits; /* keys 0..n_warps */
+  int seg_bits = 1;
+  while (seg_bits < 32 && (1ull << seg_bits) < (uint64_t)ns) ++seg_bits;
+  std::vector<uint64_t> tile0(ns + 1, 0);
+  for (uint32_t i = 0; i < ns; ++i) tile0[i + 1] = tile0[i] + ((n[i] + (1u << BT_LOG) - 1) >> BT_LOG);
+  const uint64_t ntile = tile0[ns];
+  uint64_t* slots = (uint64_t*)alloc((ntile << BT_LOG) * 8); /* worst case: every record starts a burst */
+  uint32_t* tile_cnt = (uint32_t*)alloc(ntile * 4 + 4);
+  uint64_t* tile_cnt64 = (uint64_t*)alloc(ntile * 8 + 8);
+  uint64_t* tile_off = (uint64_t*)alloc(ntile * 8 + 8);
+  const uint4** drec = (const uint4**)alloc(ns * sizeof(void*));
+  uint64_t* doff = (uint64_t*)alloc((ns + 1) * 8);
+  uint32_t* dnw = (uint32_t*)alloc(ns * 4);
+  uint64_t* start = (uint64_t*)alloc(total * 8); /* at most one burst per record */
+  unsigned long long* nb_d = (unsigned long long*)alloc(8);
+  cudaError_t e = (slots && tile_cnt && tile_cnt64 && tile_off && drec && doff && dnw && start && nb_d)
+                      ? cudaSuccess : cudaErrorMemoryAllocation;
+  if (e == cudaSuccess) e = cudaMemcpyAsync(drec, rec.data(), ns * sizeof(void*), cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(doff, off.data(), (ns + 1) * 8, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(dnw, n_warps.data(), ns * 4, cudaMemcpyHostToDevice, st);
+  for (uint32_t i = 0; i < ns && e == cudaSuccess; ++i)
+    if (n[i])
+      burst_head_kernel<<<grid_for(((n[i] + (1u << BT_LOG) - 1) >> BT_LOG) * 32, 256), 256, 0, st>>>(
+          rec[i], n[i], n_warps[i], off[i], tile0[i], slots, tile_cnt);
+  if (e == cudaSuccess) {
+    widen_kernel<<<grid_for(ntile, 256), 256, 0, st>>>(tile_cnt, ntile, tile_cnt64);
+    size_t tmp = 0;
+    cub::DeviceScan::InclusiveSum(nullptr, tmp, tile_cnt64, tile_off + 1, (int64_t)ntile, st);
+    void* dt = alloc(tmp);
+    if (!dt) e = cudaErrorMemoryAllocation;
+    else {
+      e = cudaMemsetAsync(tile_off, 0, 8, st);
+      if (e == cudaSuccess) e = cub::DeviceScan::InclusiveSum(dt, tmp, tile_cnt64, tile_off + 1, (int64_t)ntile, st);
+    }
+  }
+  if (e == cudaSuccess) {
+    burst_gather_kernel<<<grid_for(ntile * 32, 256), 256, 0, st>>>(slots, tile_cnt, tile_off, ntile, start);
+    e = cudaMemcpyAsync(nb_d, tile_off + ntile, 8, cudaMemcpyDeviceToDevice, st);
+  }
+  unsigned long long nb = 0;
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&nb, nb_d, 8, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  BucketArgs a{drec, doff, dnw, ns, warp_bits};
+  if (e == cudaSuccess) {
+    unsigned long long* key = (unsigned long long*)alloc(nb * 8);
+    unsigned long long* key2 = (unsigned long long*)alloc(nb * 8);
+    uint32_t* id = (uint32_t*)alloc(nb * 4);
+    uint32_t* sid = (uint32_t*)alloc(nb * 4);
+    uint64_t* len = (uint64_t*)alloc(nb * 8);
+    uint64_t* slen = (uint64_t*)alloc(nb * 8);
+    const uint4** ptr = (const uint4**)alloc(nb * sizeof(void*));
+    const uint4** sptr = (const uint4**)alloc(nb * sizeof(void*));
+    out->bsrc = (uint64_t*)owl_dev_alloc(nb * 8);
+    out->bdst = (uint64_t*)owl_dev_alloc(nb * 8);
+    out->out = (uint4*)owl_dev_alloc(total * 16);
+    out->nb = nb;
+    if (!key || !key2 || !id || !sid || !len || !slen || !ptr || !sptr || !out->bsrc || !out->bdst || !out->out)
+      e = cudaErrorMemoryAllocation;
+    if (e == cudaSuccess) {
+      burst_key_kernel<<<grid_for(nb, 256), 256, 0, st>>>(a, start, nb_d, key, id, len, ptr);
+      size_t tmp = 0;
+      const int bits = (int)warp_bits + seg_bits;
+      cub::DeviceRadixSort::SortPairs(nullptr, tmp, key, key2, id, sid, (int64_t)nb, 0, bits, st);
+      void* dt = alloc(tmp);
+      if (!dt) e = cudaErrorMemoryAllocation;
+      else e = cub::DeviceRadixSort::SortPairs(dt, tmp, key, key2, id, sid, (int64_t)nb, 0, bits, st);
+    }
+    if (e == cudaSuccess) {
+      burst_sorted_kernel<<<grid_for(nb, 256), 256, 0, st>>>(sid, start, len, ptr, nb_d, slen, out->bsrc, sptr);
+      size_t tmp = 0;
+      cub::DeviceScan::ExclusiveSum(nullptr, tmp, slen, out->bdst, (int64_t)nb, st);
+      void* dt = alloc(tmp);
+      if (!dt) e = cudaErrorMemoryAllocation;
+      else e = cub::DeviceScan::ExclusiveSum(dt, tmp, slen, out->bdst, (int64_t)nb, st);
+    }
+    if (e == cudaSuccess)
+      burst_copy_kernel<<<grid_for((nb + 3) / 4 * 32, 256), 256, 0, st>>>(sptr, slen, out->bdst, nb_d, out->out);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st); /* the scratch (drec, slen) is freed below */
+  }
+  for (void* p : scratch) owl_dev_free(p);
+  if (e != cudaSuccess) owl_bucketed_free(out);
+  return e == cudaSuccess ? cudaGetLastError() : e;
+}
+
+cudaError_t owl_first_bad_record(const BucketedSet& b, uint32_t seg, uint32_t n_warps, unsigned long long* idx_code,
+                                 cudaStream_t st) {
   unsigned long long* d = (unsigned long long*)owl_dev_alloc(8);
   if (!d) return cudaErrorMemoryAllocation;
+  const uint64_t n = b.off[seg + 1] - b.off[seg];
   cudaError_t e = cudaMemsetAsync(d, 0xFF, 8, st);
-  if (e == cudaSuccess && n) first_bad_kernel<<<grid_for(n, 256), 256, 0, st>>>(rec, perm, n, n_warps, d);
+  if (e == cudaSuccess && n)
+    first_bad_kernel<<<grid_for(n, 256), 256, 0, st>>>(b.out + b.off[seg], n, n_warps, b.bsrc, b.bdst, b.nb, b.off[seg], d);
   if (e == cudaSuccess) e = cudaMemcpyAsync(idx_code, d, 8, cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   owl_dev_free(d);
   return e;
-}
-
-cudaError_t owl_bucket_by_warp(const uint4* rec, uint64_t n, uint32_t n_warps, uint4* out, uint64_t* perm,
-                               cudaStream_t st) {
-  if (!n) return cudaSuccess;
-  uint32_t* gw = (uint32_t*)owl_dev_alloc(n * 4);
-  uint32_t* gw2 = (uint32_t*)owl_dev_alloc(n * 4);
-  uint64_t* idx = (uint64_t*)owl_dev_alloc(n * 8);
-  cudaError_t e = (gw && gw2 && idx) ? cudaSuccess : cudaErrorMemoryAllocation;
-  void* dt = nullptr;
-  if (e == cudaSuccess) {
-    bucket_keys_kernel<<<grid_for(n, 256), 256, 0, st>>>(rec, n, n_warps, gw, idx);
-    int bits = 1;
-    while (bits < 32 && (1ull << bits) <= (uint64_t)n_warps) ++bits; /* keys 0..n_warps */
-    size_t tmp = 0;
-    cub::DeviceRadixSort::SortPairs(nullptr, tmp, gw, gw2, idx, perm, (int64_t)n, 0, bits, st);
-    dt = owl_dev_alloc(tmp);
-    if (!dt) e = cudaErrorMemoryAllocation;
-    else e = cub::DeviceRadixSort::SortPairs(dt, tmp, gw, gw2, idx, perm, (int64_t)n, 0, bits, st);
-    if (e == cudaSuccess) gather_records_kernel<<<grid_for(n, 256), 256, 0, st>>>(rec, perm, n, out);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  }
-  owl_dev_free(gw); owl_dev_free(gw2); owl_dev_free(idx); owl_dev_free(dt);
-  return e == cudaSuccess ? cudaGetLastError() : e;
 }

@@ -164,6 +164,24 @@ def device_records(p: Params, run: int, seq: int, device=None, stream=None):
     return buf[: n * 16], n
 
 
+def device_interleave(buf, n: int, burst: int = 32):
+    """Channel-order variant of a warp-major device buffer (same order as interleave(): bursts of `burst` records
+    per warp, warps round-robin), built with torch on the device (bench / test infrastructure).  Returns a new
+    uint8 tensor of 16*n bytes."""
+    import torch
+    if n == 0:
+        return buf.clone()
+    rec = buf[: n * 16].view(torch.int32).view(n, 4)
+    g = rec[:, 2].to(torch.int64) & 0xFFFFFFFF
+    pos = torch.arange(n, device=buf.device, dtype=torch.int64)
+    first = torch.ones(n, dtype=torch.bool, device=buf.device)
+    first[1:] = g[1:] != g[:-1]
+    start = torch.cummax(torch.where(first, pos, torch.zeros_like(pos)), 0).values  # start of each record's warp
+    q = (pos - start) // burst
+    order = torch.argsort(q * (1 << 33) + start, stable=True)  # round q, then the warps in stream order
+    return rec[order].contiguous().view(torch.uint8).view(-1)
+
+
 def interleave(rec: np.ndarray, burst: int = 32) -> np.ndarray:
     """Channel-order variant (reading R17): bursts of `burst` records per warp, warps round-robin.
     Pure reordering: each warp's records keep their relative order."""
