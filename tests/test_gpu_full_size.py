@@ -43,7 +43,7 @@ def _chunks(p):
     return [runs[i:i + k] for i in range(0, len(runs), k)]
 
 
-def _build_full(ctx, p):
+def _build_full(ctx, p, channel_order=False):
     ev = {0: None, 1: None}
     n_rec = 0
     for chunk in _chunks(p):
@@ -51,7 +51,10 @@ def _build_full(ctx, p):
         for r in chunk:
             for m in tracegen.run_segments(p, r):
                 buf, n = tracegen.device_records(p, r, m.seq)
-                segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, n))
+                if channel_order:
+                    buf = tracegen.device_interleave(buf, n)
+                segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, buf, n,
+                                        flags=0 if channel_order else api.OWL_SEG_WARP_MAJOR))
                 n_rec += n
         torch.cuda.synchronize()
         ctx.ingest(segs)
@@ -71,13 +74,15 @@ def _build_full(ctx, p):
     return ev[0], ev[1], n_rec
 
 
-@pytest.mark.parametrize("cfg", [1, 2, 3, 4, 5])
-def test_full_size_parity(cfg):
+@pytest.mark.parametrize("cfg,channel_order", [(1, False), (2, False), (3, False), (4, False), (5, False), (2, True)])
+def test_full_size_parity(cfg, channel_order):
+    """(2, True): the bench's workload in a tracer channel's order (bursts of 32, warps round-robin) gives the
+    same A-DCFGs (reading R17), through the burst bucketing."""
     doc, o_ks, o_leaks = _fixture(cfg)
     p = tracegen.Params.preset(cfg)
     assert (p.runs_fix, p.runs_rnd) == (doc["runs_fix"], doc["runs_rnd"])
     ctx = api.Context(0)
-    ef, er, n_rec = _build_full(ctx, p)
+    ef, er, n_rec = _build_full(ctx, p, channel_order)
     assert n_rec == doc["records"]
     bf, br = ef.export(), er.export()
     assert (len(bf), len(br)) == (doc["e_fix_bytes"], doc["e_rnd_bytes"])
