@@ -592,7 +592,7 @@ void unpack(int t, const Key128& k, uint32_t& slot, uint32_t& a, uint32_t& b, ui
 
 OWL_API const char* owl_last_error(void) { return g_err.c_str(); }
 OWL_API const char* owl_version(void) { return "owl-b200 0.1 (sm_100a)"; }
-OWL_API void owl_free(void* p) { free(p); }
+OWL_API void owl_free(void* p) { owl_host_free(p); }
 
 OWL_API owl_status owl_ctx_create(int cuda_device, owl_ctx** out) {
   if (!out) return fail(OWL_ERR_INVALID_ARG, "out is NULL");
@@ -966,7 +966,7 @@ OWL_API owl_status owl_filter_inputs(owl_ctx* ctx, const uint32_t* runs, size_t 
         owl_diff* rows = nullptr;
         uint64_t nd = 0;
         CUDA_TRY(owl_diff_rows(a->sorted, g->sorted, T_NUM, &rows, &nd, 0, ctx->stream), "filter: compare");
-        free(rows);
+        owl_host_free(rows);
         same = nd == 0;
       }
       if (same) {

@@ -176,6 +176,8 @@ cudaError_t owl_absorb_cells(const DevTable* tabs, const ExchangeCell* cells, ui
 void* owl_dev_alloc(size_t bytes);
 void owl_dev_free(void* p);
 void owl_dev_trim(int device); /* return cached blocks to CUDA */
+void* owl_host_alloc(size_t bytes); /* pinned (cached) host block for result rows; owl_host_free releases it */
+void owl_host_free(void* p);        /* pinned pool block or plain malloc block */
 
 /* host-side key helpers */
 static inline uint64_t owl_mix64(uint64_t x) {

@@ -189,6 +189,53 @@ void* owl_dev_alloc(size_t bytes) {
   return p;
 }
 
+/* Pinned host blocks for result rows (diff rows can be millions): a D2H copy into pinned memory runs at PCIe
+   speed, into fresh pageable memory it is staged and page-faulted.  Blocks are cached by power-of-two size
+   class (at most kHostCache bytes kept); owl_host_free returns them, and frees plain malloc blocks. */
+namespace {
+std::mutex g_host_mu;
+std::map<size_t, std::vector<void*>> g_host_pool;
+std::map<void*, size_t> g_host_live;
+size_t g_host_cached = 0;
+const size_t kHostCache = 4ull << 30;
+}  // namespace
+
+void* owl_host_alloc(size_t bytes) {
+  size_t sz = 4096;
+  while (sz < bytes) sz <<= 1;
+  std::lock_guard<std::mutex> lk(g_host_mu);
+  auto it = g_host_pool.find(sz);
+  void* p = nullptr;
+  if (it != g_host_pool.end() && !it->second.empty()) {
+    p = it->second.back();
+    it->second.pop_back();
+    g_host_cached -= sz;
+  } else if (cudaMallocHost(&p, sz) != cudaSuccess) {
+    cudaGetLastError();
+    return malloc(bytes ? bytes : 1); /* not pinned: owl_host_free frees it */
+  }
+  g_host_live[p] = sz;
+  return p;
+}
+
+void owl_host_free(void* p) {
+  if (!p) return;
+  std::lock_guard<std::mutex> lk(g_host_mu);
+  auto it = g_host_live.find(p);
+  if (it == g_host_live.end()) {
+    free(p);
+    return;
+  }
+  const size_t sz = it->second;
+  g_host_live.erase(it);
+  if (g_host_cached + sz <= kHostCache) {
+    g_host_pool[sz].push_back(p);
+    g_host_cached += sz;
+  } else {
+    cudaFreeHost(p);
+  }
+}
+
 void owl_dev_free(void* p) {
   if (!p) return;
   std::lock_guard<std::mutex> lk(g_pool_mu);
@@ -472,14 +519,14 @@ cudaError_t owl_diff_rows(const SortedTable* A, const SortedTable* B, int ntab, 
   if (e == cudaSuccess) e = cudaMemcpyAsync(&total, base + ntab, 8, cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   if (e == cudaSuccess) {
-    *rows = (owl_diff*)malloc((total + extra_rows + 1) * sizeof(owl_diff));
+    *rows = (owl_diff*)owl_host_alloc((total + extra_rows + 1) * sizeof(owl_diff));
     if (!*rows) e = cudaErrorMemoryAllocation;
   }
   if (e == cudaSuccess && total) e = cudaMemcpyAsync(*rows, drows, total * sizeof(owl_diff), cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   for (void* p : scratch) owl_dev_free(p);
   if (e != cudaSuccess) {
-    free(*rows);
+    owl_host_free(*rows);
     *rows = nullptr;
     return e;
   }
