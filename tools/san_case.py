@@ -13,8 +13,12 @@ import torch  # noqa: E402
 import tracegen  # noqa: E402
 from paper_conf_dsn_zhaoxcqzj24_b200 import api  # noqa: E402
 
+CASES = ((1, 1, 10, 10, False), (2, 64, 2, 2, False), (2, 64, 1, 1, True), (9, 16, 2, 3, False))
+if os.environ.get("SAN_CASES"):  # e.g. "3:8:2:2,5:16:2:2" = config:grid_div:runs_fix:runs_rnd (warp-major)
+    CASES = tuple(tuple(int(x) for x in c.split(":")) + (False,) for c in os.environ["SAN_CASES"].split(","))
+
 ctx = api.Context(0)
-for cfg, div, nf, nr, inter in ((1, 1, 10, 10, False), (2, 64, 2, 2, False), (2, 64, 1, 1, True), (9, 16, 2, 3, False)):
+for cfg, div, nf, nr, inter in CASES:
     p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=nf, runs_rnd=nr)
     segs = []
     for r in range(p.n_runs):
