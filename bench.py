@@ -199,6 +199,7 @@ def e2e_leg(args, p, api, tracegen, dev, stream, n_runs_e2e, my_runs, world=1, r
     import torch
     import torch.distributed as dist
     ctx = api.Context(dev.index)
+    ctx.set_config(channel_order=CHANNEL_MODES[args.channel_mode])
     base_run = 1 << 20  # run ids disjoint from the device-resident leg
     runs_f = [r for r in my_runs if tracegen.run_class(p, r) == 0][: n_runs_e2e // 2]
     runs_r = [r for r in my_runs if tracegen.run_class(p, r) == 1][: n_runs_e2e // 2]
@@ -318,6 +319,7 @@ def run_ours(args):
     if args.runs:
         my_runs = my_runs[: args.runs]
     ctx = api.Context(local)
+    ctx.set_config(channel_order=CHANNEL_MODES[args.channel_mode])
     stream = torch.cuda.current_stream(dev)
     chunks = _chunks(tracegen, p, my_runs, args.hbm_budget_gb * 1e9)
     resident = len(chunks) == 1
@@ -479,7 +481,8 @@ def run_ours(args):
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": mode,
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
         "config": {"workload": tracegen.CONFIG_NAMES[cfg] + (" (channel order)" if args.channel_order else ""),
-                   "record_order": "channel (bursts of 32, warps round-robin)" if args.channel_order else "warp-major",
+                   "record_order": ("channel (bursts of 32, warps round-robin; %s)" % args.channel_mode)
+                   if args.channel_order else "warp-major",
                    "runs_per_gpu": len(my_runs), "runs_total": p.n_runs,
                    "records_per_gpu": n_records, "bytes_per_gpu": 16 * n_records,
                    "l2": "inputs (%.1f GB) >> 126 MB L2; no flush needed" % (16 * n_records / 1e9),
@@ -527,6 +530,9 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
+CHANNEL_MODES = {"auto": 0, "copy": 1, "inplace": 2}  # owl_config.channel_order
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -546,6 +552,8 @@ def main():
     ap.add_argument("--e2e-gb", type=float, default=8.0, help="pinned host bytes of the e2e leg's runs (bound)")
     ap.add_argument("--channel-order", action="store_true",
                     help="records in a tracer channel's order (bursts of 32 per warp, warps round-robin; N2)")
+    ap.add_argument("--channel-mode", default="auto", choices=sorted(CHANNEL_MODES),
+                    help="channel-order bucketing: copy to warp-major, fold in place, or auto (owl_config.channel_order)")
     ap.add_argument("--dump", default="", help="rank 0 writes the last step's diff / leak rows here (tests)")
     args = ap.parse_args()
     import __graft_entry__

@@ -109,8 +109,16 @@ typedef struct {
                                default) = joint counts c_ij; OWL_HCF_ROW_NORMALIZED (1) = the elements
                                a_ij = c_ij / x_i of the transition matrix A (Eqs. 7-8).  Other values:
                                OWL_ERR_INVALID_ARG from owl_ctx_set_config.                          */
-  uint32_t _reserved;
+  uint32_t channel_order;   /* segments without OWL_SEG_WARP_MAJOR (a tracer channel's order, reading R17,
+                               P:L183, L211) are bucketed by warp on the device, by bursts
+                               of consecutive records of one warp.  OWL_CHANNEL_AUTO (0, default): copy the
+                               bursts to a warp-major buffer when it fits in free device memory, else fold
+                               them in place; OWL_CHANNEL_COPY (1): always copy (16 B per record of
+                               scratch, the faster fold); OWL_CHANNEL_IN_PLACE (2): never copy, the fold
+                               reads every record through the burst index (needs every segment < 2^32
+                               records, else the copy is used).  Other values: OWL_ERR_INVALID_ARG.      */
 } owl_config;
+enum { OWL_CHANNEL_AUTO = 0u, OWL_CHANNEL_COPY = 1u, OWL_CHANNEL_IN_PLACE = 2u };
 
 /* H_cf readings.  R2 weights each (src, dst) cell of a node by a_ij = c_ij / x_i, with
    x_i = sum_j c_ij the src count of Eq. 5, and tests F(t) = sum_{cells <= t} a / k (k = number of srcs,

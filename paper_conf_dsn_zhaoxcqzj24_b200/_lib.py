@@ -17,7 +17,7 @@ class OwlSegment(ctypes.Structure):
 
 class OwlConfig(ctypes.Structure):
     _fields_ = [("addr_capacity", u64), ("cf_capacity", u64), ("max_regrow", u32), ("fold_ctas_per_sm", u32),
-                ("host_chunk_bytes", u64), ("hcf_reading", u32), ("_reserved", u32)]
+                ("host_chunk_bytes", u64), ("hcf_reading", u32), ("channel_order", u32)]
 
 
 class OwlAdcfgInfo(ctypes.Structure):

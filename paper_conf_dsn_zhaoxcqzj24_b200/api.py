@@ -19,6 +19,7 @@ from . import _lib
 
 OWL_FIXED, OWL_RANDOM = 0, 1
 OWL_SEG_WARP_MAJOR, OWL_SEG_HOST_RECORDS = 1, 2
+OWL_CHANNEL_AUTO, OWL_CHANNEL_COPY, OWL_CHANNEL_IN_PLACE = 0, 1, 2  # owl_config.channel_order (N2)
 
 DIFF_DTYPE = np.dtype([("table", "<u4"), ("slot", "<u4"), ("bb", "<u4"), ("ins", "<u4"), ("j", "<u4"),
                        ("prev", "<u4"), ("next", "<u4"), ("_pad", "<u4"), ("x", "<u8"), ("count_a", "<u8"),
@@ -152,10 +153,11 @@ class Context:
             self.h = None
 
     def set_config(self, addr_capacity=0, cf_capacity=0, max_regrow=0, fold_ctas_per_sm=0, host_chunk_bytes=0,
-                   hcf_reading=0):
-        """owl_ctx_set_config.  hcf_reading: 0 = joint counts (R1), 1 = row-normalized A (R2, Eq. 7)."""
+                   hcf_reading=0, channel_order=0):
+        """owl_ctx_set_config.  hcf_reading: 0 = joint counts (R1), 1 = row-normalized A (R2, Eq. 7).
+        channel_order: 0 auto, 1 copy to warp-major, 2 fold in place through the burst index (include/owl.h)."""
         cfg = _lib.OwlConfig(addr_capacity, cf_capacity, max_regrow, fold_ctas_per_sm, host_chunk_bytes,
-                             hcf_reading, 0)
+                             hcf_reading, channel_order)
         _check(_lib.load().owl_ctx_set_config(self.h, ctypes.byref(cfg)))
 
     def ingest(self, segments, stream=None):

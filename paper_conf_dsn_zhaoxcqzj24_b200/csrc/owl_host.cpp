@@ -235,6 +235,7 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
   *overflow = 0;
   const uint32_t tile_shift = getenv("OWL_TILE_SHIFT") ? (uint32_t)atoi(getenv("OWL_TILE_SHIFT")) : 15u; /* tile sweep: profiles/r01_v4_ab.txt */
   std::vector<FoldSeg> fs(plan.size());
+  std::vector<FoldBurst> fb(plan.size(), FoldBurst{nullptr, nullptr, nullptr, 0}); /* in-place channel order */
   std::vector<void*> scratch;
   std::vector<BucketedSet> sets; /* channel-order segments, bucketed per launch */
   std::vector<std::pair<uint32_t, uint32_t>> bucketed(plan.size(), {~0u, 0u}); /* (set, position) */
@@ -350,55 +351,95 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
         bi.push_back(i);
       }
       if (!bi.empty()) {
+        /* copy to a warp-major buffer (the faster fold) or walk the burst index in place (no 16 B per record of
+           scratch): owl_config.channel_order; AUTO copies when it fits with 1 GiB to spare */
+        uint64_t tot = 0;
+        bool fits = true;
+        for (uint64_t x : bn) { tot += x; fits = fits && x < (1ull << 32); }
+        bool inplace = ctx->cfg.channel_order == OWL_CHANNEL_IN_PLACE;
+        if (ctx->cfg.channel_order == OWL_CHANNEL_AUTO) {
+          size_t fr = 0, tt = 0;
+          cudaMemGetInfo(&fr, &tt);
+          inplace = tot * 32 + (1ull << 30) > fr; /* the copy (16 B / record) next to the burst heads' scratch */
+        }
+        inplace = inplace && fits;
         sets.emplace_back();
-        const cudaError_t e = owl_bucket_segments(brec, bn, bw, &sets.back(), st);
+        const cudaError_t e = owl_bucket_segments(brec, bn, bw, &sets.back(), st, !inplace);
         if (e != cudaSuccess) { status = cuda_fail(e, "fold: bucketing"); break; }
+        const BucketedSet& bs = sets.back();
         for (size_t k = 0; k < bi.size(); ++k) {
-          fs[bi[k]].rec = sets.back().out + sets.back().off[k];
+          if (inplace) {
+            FoldBurst& f = fb[bi[k]];
+            f.bvs = bs.bvs + bs.bfirst[k];
+            f.bpo = bs.bpo + bs.bfirst[k];
+            f.bk = bs.bk + bs.bfirst[k];
+            f.nb = bs.bfirst[k + 1] - bs.bfirst[k];
+          } else {
+            fs[bi[k]].rec = bs.out + bs.off[k];
+          }
           bucketed[bi[k]] = {(uint32_t)sets.size() - 1, (uint32_t)k};
         }
       }
     }
-    /* work items: (segment, tile of 2^tile_shift records), one range per segment */
-    std::vector<FoldSeg> lsegs;
-    std::vector<FoldGroup> groups;
-    uint64_t items = 0, lrec = 0;
-    for (size_t i : launches[w]) {
-      const uint64_t ntile = (fs[i].n + (1ull << tile_shift) - 1) >> tile_shift;
-      if (!ntile) continue;
-      FoldGroup g;
-      g.item0 = items;
-      g.first_seg = (uint32_t)lsegs.size();
-      g._pad = 0;
-      lsegs.push_back(fs[i]);
-      groups.push_back(g);
-      items += ntile;
-      lrec += fs[i].n;
+    /* work items: (segment, tile of 2^tile_shift records), one range per segment; in-place channel-order segments
+       (bursts walked through their index) get their own launch of fold_burst_kernel, items of 2^burst_shift bursts */
+    const uint32_t burst_shift = getenv("OWL_BURST_SHIFT") ? (uint32_t)atoi(getenv("OWL_BURST_SHIFT")) : 10u;
+    cudaError_t e = cudaSuccess;
+    bool any = false;
+    for (int mode = 0; mode < 2 && e == cudaSuccess; ++mode) {
+      std::vector<FoldSeg> lsegs;
+      std::vector<FoldBurst> lbursts;
+      std::vector<FoldGroup> groups;
+      uint64_t items = 0;
+      const uint32_t shift = mode ? burst_shift : tile_shift;
+      for (size_t i : launches[w]) {
+        if ((fb[i].bvs != nullptr) != (mode == 1)) continue;
+        const uint64_t units = mode ? fb[i].nb : fs[i].n;
+        const uint64_t ntile = (units + (1ull << shift) - 1) >> shift;
+        if (!ntile) continue;
+        FoldGroup g;
+        g.item0 = items;
+        g.first_seg = (uint32_t)lsegs.size();
+        g._pad = 0;
+        lsegs.push_back(fs[i]);
+        lbursts.push_back(fb[i]);
+        groups.push_back(g);
+        items += ntile;
+      }
+      if (!items) continue;
+      FoldBurst* dbursts = nullptr;
+      if (mode) {
+        dbursts = (FoldBurst*)owl_dev_alloc(lbursts.size() * sizeof(FoldBurst) + 16);
+        if (!dbursts) { e = cudaErrorMemoryAllocation; break; }
+        scratch.push_back(dbursts);
+        cudaMemcpyAsync(dbursts, lbursts.data(), lbursts.size() * sizeof(FoldBurst), cudaMemcpyHostToDevice, st);
+      }
+      FoldSeg* dsegs = (FoldSeg*)owl_dev_alloc(lsegs.size() * sizeof(FoldSeg) + 16);
+      FoldGroup* dgroups = (FoldGroup*)owl_dev_alloc(groups.size() * sizeof(FoldGroup) + 16);
+      if (!dsegs || !dgroups) { owl_dev_free(dsegs); owl_dev_free(dgroups); e = cudaErrorMemoryAllocation; break; }
+      scratch.push_back(dsegs);
+      scratch.push_back(dgroups);
+      cudaMemcpyAsync(dsegs, lsegs.data(), lsegs.size() * sizeof(FoldSeg), cudaMemcpyHostToDevice, st);
+      cudaMemcpyAsync(dgroups, groups.data(), groups.size() * sizeof(FoldGroup), cudaMemcpyHostToDevice, st);
+      cudaMemsetAsync(&ctx->d_status->tile_counter, 0, sizeof(unsigned long long), st); /* the launch's work counter */
+      FoldArgs a;
+      a.segs = dsegs;
+      a.groups = dgroups;
+      a.n_groups = (uint32_t)groups.size();
+      a.tile_shift = shift;
+      a.n_items = items;
+      for (int t = 0; t < T_NUM; ++t) a.tab[t] = tab[t];
+      a.status = ctx->d_status;
+      a.mode = getenv("OWL_FOLD_MODE") ? (uint32_t)atoi(getenv("OWL_FOLD_MODE")) : 0u;
+      a.vmap = vmap;
+      if (!any) cudaEventRecord(ctx->ev0, st);
+      any = true;
+      e = mode ? owl_launch_fold_bursts(a, dbursts, grid, st) : owl_launch_fold(a, grid, st);
     }
-    if (!items) {
+    if (!any && e == cudaSuccess) {
       if (w >= 1) cudaEventRecord(freed[(w - 1) & 1], st);
       continue;
     }
-    FoldSeg* dsegs = (FoldSeg*)owl_dev_alloc(lsegs.size() * sizeof(FoldSeg) + 16);
-    FoldGroup* dgroups = (FoldGroup*)owl_dev_alloc(groups.size() * sizeof(FoldGroup) + 16);
-    if (!dsegs || !dgroups) { owl_dev_free(dsegs); owl_dev_free(dgroups); status = fail(OWL_ERR_OUT_OF_MEMORY, "fold: segment table"); break; }
-    scratch.push_back(dsegs);
-    scratch.push_back(dgroups);
-    cudaMemcpyAsync(dsegs, lsegs.data(), lsegs.size() * sizeof(FoldSeg), cudaMemcpyHostToDevice, st);
-    cudaMemcpyAsync(dgroups, groups.data(), groups.size() * sizeof(FoldGroup), cudaMemcpyHostToDevice, st);
-    cudaMemsetAsync(&ctx->d_status->tile_counter, 0, sizeof(unsigned long long), st); /* the launch's work counter */
-    FoldArgs a;
-    a.segs = dsegs;
-    a.groups = dgroups;
-    a.n_groups = (uint32_t)groups.size();
-    a.tile_shift = tile_shift;
-    a.n_items = items;
-    for (int t = 0; t < T_NUM; ++t) a.tab[t] = tab[t];
-    a.status = ctx->d_status;
-    a.mode = getenv("OWL_FOLD_MODE") ? (uint32_t)atoi(getenv("OWL_FOLD_MODE")) : 0u;
-    a.vmap = vmap;
-    cudaEventRecord(ctx->ev0, st);
-    cudaError_t e = owl_launch_fold(a, grid, st);
     cudaEventRecord(ctx->ev1, st);
     if (w >= 1) cudaEventRecord(freed[(w - 1) & 1], st);
     if (e == cudaSuccess && launches.size() > 1) e = cudaEventSynchronize(ctx->ev1); /* per-launch timing */
@@ -409,7 +450,6 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
       fold_ms += ms;
     }
     ++launched;
-    (void)lrec;
   }
   cudaError_t e = status == OWL_OK ? cudaMemcpyAsync(&hs, ctx->d_status, sizeof hs, cudaMemcpyDeviceToHost, st)
                                    : cudaSuccess;
@@ -445,11 +485,15 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
     /* An overflowed pass stopped early: its reports are incomplete, the regrown pass decides.  A segment that
        is flagged warp-major but is not (a warp seen twice, or records the warp walk did not cover exactly once)
        is reported first: walking it from the middle of a warp produces malformed-record artifacts. */
+    /* (bucketed channel-order segments are warp-major by construction: a walk mismatch there comes from records
+       with out-of-range gwarps, which a malformed-record report already covers) */
+    const bool reported = hs.first_error != ~0ull;
     size_t bad_walk = plan.size();
     for (size_t i = 0; i < plan.size() && bad_walk == plan.size(); ++i)
-      if (walked_h[i] != plan[i].s.n_records) bad_walk = i;
+      if (walked_h[i] != plan[i].s.n_records && !(reported && bucketed[i].first != ~0u)) bad_walk = i;
+    const uint32_t nwm_seg = (uint32_t)(hs.not_warp_major >> 32);
     if (hs.overflow) {
-    } else if (hs.not_warp_major != ~0ull) {
+    } else if (hs.not_warp_major != ~0ull && !(reported && nwm_seg < plan.size() && bucketed[nwm_seg].first != ~0u)) {
       const uint32_t si = (uint32_t)(hs.not_warp_major >> 32);
       status = fail(OWL_ERR_INVALID_ARG,
                     "segment (run %u, seq %u) is flagged OWL_SEG_WARP_MAJOR but warp %u's records are not contiguous",
@@ -632,6 +676,8 @@ OWL_API owl_status owl_ctx_set_config(owl_ctx* ctx, const owl_config* cfg) {
   if (!ctx) return fail(OWL_ERR_INVALID_ARG, "ctx is NULL");
   if (cfg && cfg->hcf_reading > OWL_HCF_ROW_NORMALIZED)
     return fail(OWL_ERR_INVALID_ARG, "hcf_reading must be OWL_HCF_COUNTS or OWL_HCF_ROW_NORMALIZED");
+  if (cfg && cfg->channel_order > OWL_CHANNEL_IN_PLACE)
+    return fail(OWL_ERR_INVALID_ARG, "channel_order must be OWL_CHANNEL_AUTO, OWL_CHANNEL_COPY or OWL_CHANNEL_IN_PLACE");
   if (cfg) ctx->cfg = *cfg;
   else ctx->cfg = owl_config{};
   for (int t = 0; t < T_NUM; ++t) ctx->cap_hint[t] = 0;

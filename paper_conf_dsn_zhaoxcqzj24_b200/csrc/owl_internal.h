@@ -81,6 +81,16 @@ struct FoldSeg {
   uint32_t _pad;
 };
 
+/* A channel-order segment walked in place (N2, fold_burst_kernel): its bursts in warp-major order (stable by stream
+   position within a warp).  Burst k starts at virtual (warp-major) record bvs[k] and at physical record bpo[k] of
+   FoldSeg::rec; bk[k] = its gwarp clamped to n_warps; nb bursts (FoldSeg::n = its records). */
+struct FoldBurst {
+  const uint32_t* bvs;
+  const uint32_t* bpo;
+  const uint32_t* bk;
+  uint64_t nb;
+};
+
 /* A work item of the fold is (segment, tile position p): one warp folds the traced warps starting in tile p.
    The items of segment first_seg are item0 .. item0 + its number of tiles - 1. */
 struct FoldGroup {
@@ -103,6 +113,8 @@ struct FoldArgs {
 
 /* ---- launchers (owl_fold.cu, owl_tables.cu, owl_ks.cu, owl_exchange.cu) ---- */
 cudaError_t owl_launch_fold(const FoldArgs& a, int grid, cudaStream_t st);
+/* in-place channel-order segments: bursts[i] describes a.segs[i] (owl_fold_burst.cu) */
+cudaError_t owl_launch_fold_bursts(const FoldArgs& a, const FoldBurst* bursts, int grid, cudaStream_t st);
 int owl_fold_ctas_per_sm();
 size_t owl_fold_scratch_bytes(int grid);
 int owl_fold_max_bbs(); /* distinct BBs one traced warp may visit */
@@ -136,14 +148,23 @@ cudaError_t owl_tables_fingerprint(const SortedTable* tabs, int ntab, unsigned l
    warp-major order at out + off[s]; per sorted burst, its source start (global index in the concatenation of the
    callers' segments) and its destination start in out. */
 struct BucketedSet {
-  uint4* out = nullptr;
+  uint4* out = nullptr;     /* copy mode: the segments' records in warp-major order, back to back */
   uint64_t* bsrc = nullptr;
   uint64_t* bdst = nullptr;
   uint64_t nb = 0;
   std::vector<uint64_t> off;
+  /* in-place mode (out == nullptr): per sorted burst, segment-relative virtual start / physical start / clamped
+     gwarp (u32: every segment < 2^32 records), and each segment's first sorted burst (bfirst[ns] = nb) */
+  uint32_t* bvs = nullptr;
+  uint32_t* bpo = nullptr;
+  uint32_t* bk = nullptr;
+  std::vector<uint64_t> bfirst;
+  std::vector<const uint4*> rec; /* the callers' (or staged) segment arrays */
 };
+/* copy = false: the in-place burst index only (no warp-major copy); requires every segment < 2^32 records */
 cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std::vector<uint64_t>& n,
-                                const std::vector<uint32_t>& n_warps, BucketedSet* out, cudaStream_t st);
+                                const std::vector<uint32_t>& n_warps, BucketedSet* out, cudaStream_t st,
+                                bool copy = true);
 void owl_bucketed_free(BucketedSet* b);
 /* the first malformed record (caller's index in segment seg << 3 | KERR code, ~0 if none) of a bucketed set */
 cudaError_t owl_first_bad_record(const BucketedSet& b, uint32_t seg, uint32_t n_warps, unsigned long long* idx_code,

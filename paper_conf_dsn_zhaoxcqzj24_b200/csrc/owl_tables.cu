@@ -724,18 +724,25 @@ __device__ __forceinline__ uint64_t caller_index(uint64_t d, const uint64_t* bsr
   return bsrc[lo] + (d - bdst[lo]) - seg_off;
 }
 
-__global__ void first_bad_kernel(const uint4* rec, uint64_t n, uint32_t n_warps, const uint64_t* bsrc,
-                                 const uint64_t* bdst, uint64_t nb, uint64_t seg_off, unsigned long long* out) {
+/* rec: the warp-major copy (copy mode), or nullptr with caller = the segment's own array (in-place mode: the
+   record at warp-major index i is read through its burst) */
+__global__ void first_bad_kernel(const uint4* rec, const uint4* caller, uint64_t n, uint32_t n_warps,
+                                 const uint64_t* bsrc, const uint64_t* bdst, uint64_t nb, uint64_t seg_off,
+                                 unsigned long long* out) {
+  auto at = [&](uint64_t i) -> uint4 {
+    return rec ? rec[i] : caller[caller_index(seg_off + i, bsrc, bdst, nb, seg_off)];
+  };
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t g = rec[i].z;
+    const uint32_t g = at(i).z;
     if (g >= n_warps) {
       atomicMin(out, ((unsigned long long)caller_index(seg_off + i, bsrc, bdst, nb, seg_off) << 3) | KERR_GWARP);
       continue;
     }
-    if (i > 0 && rec[i - 1].z == g) continue;
+    if (i > 0 && at(i - 1).z == g) continue;
     uint32_t cur = OWL_NONE_BB;
-    for (uint64_t k = i; k < n && rec[k].z == g; ++k) {
-      const uint4 r = rec[k];
+    for (uint64_t k = i; k < n; ++k) {
+      const uint4 r = at(k);
+      if (r.z != g) break;
       const uint32_t bb = (r.w >> 8) & 0x3FFFFu;
       uint32_t code = KERR_NONE;
       if ((r.w >> 31) == 0) {
@@ -748,18 +755,51 @@ __global__ void first_bad_kernel(const uint4* rec, uint64_t n, uint32_t n_warps,
     }
   }
 }
+
+/* in-place burst index (N2): per sorted burst its segment-relative virtual start, physical start and clamped gwarp */
+__global__ void burst_inplace_kernel(const unsigned long long* key2, const uint64_t* bsrc, const uint64_t* bdst,
+                                     const uint64_t* off, uint32_t warp_bits, const unsigned long long* nb_p,
+                                     uint32_t* bvs, uint32_t* bpo, uint32_t* bk) {
+  const uint64_t nb = *nb_p;
+  for (uint64_t b = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; b < nb; b += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long k = key2[b];
+    const uint64_t so = off[k >> warp_bits];
+    bvs[b] = (uint32_t)(bdst[b] - so);
+    bpo[b] = (uint32_t)(bsrc[b] - so);
+    bk[b] = (uint32_t)(k & ((1ull << warp_bits) - 1));
+  }
+}
+
+/* first sorted burst of every segment: lower bound of (s << warp_bits) in the sorted keys; first[ns] = nb */
+__global__ void seg_first_kernel(const unsigned long long* key2, const unsigned long long* nb_p, uint32_t ns,
+                                 uint32_t warp_bits, uint64_t* first) {
+  const uint64_t nb = *nb_p;
+  for (uint32_t s = blockIdx.x * blockDim.x + threadIdx.x; s <= ns; s += gridDim.x * blockDim.x) {
+    const unsigned long long want = (unsigned long long)s << warp_bits;
+    uint64_t lo = 0, hi = nb;
+    while (lo < hi) {
+      const uint64_t mid = (lo + hi) >> 1;
+      if (key2[mid] < want) lo = mid + 1; else hi = mid;
+    }
+    first[s] = s == ns ? nb : lo;
+  }
+}
 }  // namespace
 
 void owl_bucketed_free(BucketedSet* b) {
   owl_dev_free(b->out);
   owl_dev_free(b->bsrc);
   owl_dev_free(b->bdst);
+  owl_dev_free(b->bvs);
+  owl_dev_free(b->bpo);
+  owl_dev_free(b->bk);
   *b = BucketedSet{};
 }
 
 cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std::vector<uint64_t>& n,
-                                const std::vector<uint32_t>& n_warps, BucketedSet* out, cudaStream_t st) {
+                                const std::vector<uint32_t>& n_warps, BucketedSet* out, cudaStream_t st, bool copy) {
   *out = BucketedSet{};
+  out->rec = rec;
   const uint32_t ns = (uint32_t)rec.size();
   std::vector<uint64_t> off(ns + 1, 0);
   uint32_t maxw = 1;
@@ -827,9 +867,16 @@ cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std:
     const uint4** sptr = (const uint4**)alloc(nb * sizeof(void*));
     out->bsrc = (uint64_t*)owl_dev_alloc(nb * 8);
     out->bdst = (uint64_t*)owl_dev_alloc(nb * 8);
-    out->out = (uint4*)owl_dev_alloc(total * 16);
+    if (copy) {
+      out->out = (uint4*)owl_dev_alloc(total * 16);
+    } else {
+      out->bvs = (uint32_t*)owl_dev_alloc(nb * 4 + 4);
+      out->bpo = (uint32_t*)owl_dev_alloc(nb * 4 + 4);
+      out->bk = (uint32_t*)owl_dev_alloc(nb * 4 + 4);
+    }
     out->nb = nb;
-    if (!key || !key2 || !id || !sid || !len || !slen || !ptr || !sptr || !out->bsrc || !out->bdst || !out->out)
+    if (!key || !key2 || !id || !sid || !len || !slen || !ptr || !sptr || !out->bsrc || !out->bdst ||
+        (copy ? !out->out : (!out->bvs || !out->bpo || !out->bk)))
       e = cudaErrorMemoryAllocation;
     if (e == cudaSuccess) {
       burst_key_kernel<<<grid_for(nb, 256), 256, 0, st>>>(a, start, nb_d, key, id, len, ptr);
@@ -848,8 +895,19 @@ cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std:
       if (!dt) e = cudaErrorMemoryAllocation;
       else e = cub::DeviceScan::ExclusiveSum(dt, tmp, slen, out->bdst, (int64_t)nb, st);
     }
-    if (e == cudaSuccess)
+    if (e == cudaSuccess && copy)
       burst_copy_kernel<<<grid_for((nb + 3) / 4 * 32, 256), 256, 0, st>>>(sptr, slen, out->bdst, nb_d, out->out);
+    if (e == cudaSuccess && !copy) {
+      burst_inplace_kernel<<<grid_for(nb, 256), 256, 0, st>>>(key2, out->bsrc, out->bdst, doff, warp_bits, nb_d,
+                                                              out->bvs, out->bpo, out->bk);
+      uint64_t* dfirst = (uint64_t*)alloc((ns + 1) * 8);
+      if (!dfirst) e = cudaErrorMemoryAllocation;
+      else {
+        seg_first_kernel<<<grid_for(ns + 1, 128), 128, 0, st>>>(key2, nb_d, ns, warp_bits, dfirst);
+        out->bfirst.assign(ns + 1, 0);
+        e = cudaMemcpyAsync(out->bfirst.data(), dfirst, (ns + 1) * 8, cudaMemcpyDeviceToHost, st);
+      }
+    }
     if (e == cudaSuccess) e = cudaStreamSynchronize(st); /* the scratch (drec, slen) is freed below */
   }
   for (void* p : scratch) owl_dev_free(p);
@@ -864,7 +922,8 @@ cudaError_t owl_first_bad_record(const BucketedSet& b, uint32_t seg, uint32_t n_
   const uint64_t n = b.off[seg + 1] - b.off[seg];
   cudaError_t e = cudaMemsetAsync(d, 0xFF, 8, st);
   if (e == cudaSuccess && n)
-    first_bad_kernel<<<grid_for(n, 256), 256, 0, st>>>(b.out + b.off[seg], n, n_warps, b.bsrc, b.bdst, b.nb, b.off[seg], d);
+    first_bad_kernel<<<grid_for(n, 256), 256, 0, st>>>(b.out ? b.out + b.off[seg] : nullptr, b.rec[seg], n, n_warps,
+                                                       b.bsrc, b.bdst, b.nb, b.off[seg], d);
   if (e == cudaSuccess) e = cudaMemcpyAsync(idx_code, d, 8, cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   owl_dev_free(d);

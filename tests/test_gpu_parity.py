@@ -101,11 +101,17 @@ def test_c4_kernel_leak_parity(ctx):
     assert ef.info()["n_slots"] == 4
 
 
+@pytest.mark.parametrize("mode", [api.OWL_CHANNEL_COPY, api.OWL_CHANNEL_IN_PLACE])
 @pytest.mark.parametrize("cfg,div", [(1, 1), (2, 64), (5, 32)])
-def test_channel_order_input(ctx, cfg, div):
-    """Reading R17: interleaved (channel-order) records give the identical A-DCFG."""
+def test_channel_order_input(ctx, cfg, div, mode):
+    """Reading R17: interleaved (channel-order) records give the identical A-DCFG, whether the bursts are copied
+    to warp-major order or folded in place through the burst index (owl_config.channel_order)."""
     p = tracegen.Params.preset(cfg, grid_div=div, runs_fix=2, runs_rnd=2)
-    _build_and_compare(ctx, p, interleaved=True)
+    ctx.set_config(channel_order=mode)
+    try:
+        _build_and_compare(ctx, p, interleaved=True)
+    finally:
+        ctx.set_config()
 
 
 def test_accumulate_equals_single_build(ctx):
@@ -212,7 +218,13 @@ def test_random_traces_parity(ctx, seed):
         return
     want = oracle.build([oracle.Segment(0, 0, 0, n_warps, 10, rec)]).export()
     assert _build_one(ctx, rec, n_warps) == want
-    assert _build_one(ctx, H.interleave_random(rng, rec), n_warps, flags=0) == want
+    inter = H.interleave_random(rng, rec)
+    for mode in (api.OWL_CHANNEL_COPY, api.OWL_CHANNEL_IN_PLACE):
+        ctx.set_config(channel_order=mode)
+        try:
+            assert _build_one(ctx, inter, n_warps, flags=0) == want
+        finally:
+            ctx.set_config()
 
 
 def test_many_distinct_bbs(ctx):
@@ -433,6 +445,12 @@ def test_hcf_r2_parity(ctx, cfg, div, nf, nr):
 def test_hcf_reading_invalid(ctx):
     with pytest.raises(api.OwlError, match="OWL_ERR_INVALID_ARG"):
         ctx.set_config(hcf_reading=2)
+    ctx.set_config()
+
+
+def test_channel_order_mode_invalid(ctx):
+    with pytest.raises(api.OwlError, match="OWL_ERR_INVALID_ARG"):
+        ctx.set_config(channel_order=3)
     ctx.set_config()
 
 
