@@ -591,30 +591,33 @@ struct BucketArgs {
   uint32_t warp_bits;      /* key bits of the clamped gwarp */
 };
 
-__device__ __forceinline__ uint32_t seg_of(const BucketArgs& a, uint64_t g) {
-  uint32_t lo = 0, hi = a.n_seg; /* last segment with off <= g */
-  while (hi - lo > 1) {
-    const uint32_t mid = (lo + hi) >> 1;
-    if (a.off[mid] <= g) lo = mid; else hi = mid;
-  }
-  return lo;
-}
-
-/* burst heads of one segment, found and compacted in one streaming pass: each warp scans a tile of 1024 records
-   (32 coalesced loads of the gwarp words), keeps its heads in stream order in the tile's slot range of `slots`
-   and the count in tile_cnt; the tiles are concatenated afterwards (burst_gather_kernel) */
+/* burst heads of all the launch's channel-order segments in one streaming pass: each warp scans a tile of 1024
+   records of one segment (tile t belongs to the last segment with tile0 <= t; 32 coalesced loads of the gwarp
+   words, 8 in flight per lane), keeps its heads in stream order in the tile's slot range of `slots` with their
+   sort keys (segment, gwarp clamped to n_warps) in `skey`, and the count in tile_cnt; the tiles are concatenated
+   afterwards (burst_gather_kernel) */
 #define BT_LOG 10
-__global__ void burst_head_kernel(const uint4* rec, uint64_t n, uint32_t n_warps, uint64_t goff, uint64_t tile0,
-                                  uint64_t* slots, uint32_t* tile_cnt) {
+__global__ void burst_head_kernel(const BucketArgs a, const uint64_t* tile0, uint64_t ntile, uint64_t* slots,
+                                  unsigned long long* skey, uint32_t* tile_cnt) {
   const int lane = threadIdx.x & 31;
-  const uint64_t ntile = (n + (1u << BT_LOG) - 1) >> BT_LOG;
   const uint64_t wid = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
   const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
   for (uint64_t t = wid; t < ntile; t += nw) {
-    const uint64_t b = t << BT_LOG;
+    uint32_t lo = 0, hi = a.n_seg; /* the tile's segment */
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (tile0[mid] <= t) lo = mid; else hi = mid;
+    }
+    const uint32_t sg = lo;
+    const uint4* rec = a.rec[sg];
+    const uint64_t n = a.off[sg + 1] - a.off[sg], goff = a.off[sg];
+    const uint32_t n_warps = a.n_warps[sg];
+    const unsigned long long kseg = (unsigned long long)sg << a.warp_bits;
+    const uint64_t b = (t - tile0[sg]) << BT_LOG;
     uint32_t prev = b == 0 ? 0xFFFFFFFFu : min(__ldg(&rec[b - 1].z), n_warps);
     uint32_t cnt = 0;
-    uint64_t* out = slots + ((tile0 + t) << BT_LOG);
+    uint64_t* out = slots + (t << BT_LOG);
+    unsigned long long* kout = skey + (t << BT_LOG);
     for (int it0 = 0; it0 < (1 << BT_LOG) / 32; it0 += 8) {
       uint32_t gg[8]; /* 8 loads in flight per lane */
 #pragma unroll
@@ -630,24 +633,35 @@ __global__ void burst_head_kernel(const uint4* rec, uint64_t n, uint32_t n_warps
         if (lane == 0) left = prev;
         const bool head = i < n && (i == 0 || g != left);
         const unsigned m = __ballot_sync(0xFFFFFFFFu, head);
-        if (head) out[cnt + __popc(m & ((1u << lane) - 1))] = goff + i;
+        if (head) {
+          const uint32_t k = cnt + __popc(m & ((1u << lane) - 1));
+          out[k] = goff + i;
+          kout[k] = kseg | g;
+        }
         cnt += __popc(m);
         prev = __shfl_sync(0xFFFFFFFFu, g, 31);
       }
     }
-    if (lane == 0) tile_cnt[tile0 + t] = cnt;
+    if (lane == 0) tile_cnt[t] = cnt;
   }
 }
 
-/* concatenation of the tiles' heads (tile_off = exclusive scan of tile_cnt): global burst starts in stream order */
-__global__ void burst_gather_kernel(const uint64_t* slots, const uint32_t* tile_cnt, const uint64_t* tile_off,
-                                    uint64_t ntile, uint64_t* start) {
+/* concatenation of the tiles' heads (tile_off = exclusive scan of tile_cnt): global burst starts in stream order,
+   their sort keys, and the original burst ids (the sort's values) */
+__global__ void burst_gather_kernel(const uint64_t* slots, const unsigned long long* skey, const uint32_t* tile_cnt,
+                                    const uint64_t* tile_off, uint64_t ntile, uint64_t* start, unsigned long long* key,
+                                    uint32_t* id) {
   const int lane = threadIdx.x & 31;
   const uint64_t wid = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
   const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
   for (uint64_t t = wid; t < ntile; t += nw) {
     const uint32_t c = tile_cnt[t];
-    for (uint32_t k = lane; k < c; k += 32) start[tile_off[t] + k] = slots[(t << BT_LOG) + k];
+    const uint64_t o = tile_off[t];
+    for (uint32_t k = lane; k < c; k += 32) {
+      start[o + k] = slots[(t << BT_LOG) + k];
+      key[o + k] = skey[(t << BT_LOG) + k];
+      id[o + k] = (uint32_t)(o + k);
+    }
   }
 }
 
@@ -655,29 +669,19 @@ __global__ void widen_kernel(const uint32_t* in, uint64_t n, uint64_t* out) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) out[i] = in[i];
 }
 
-__global__ void burst_key_kernel(const BucketArgs a, const uint64_t* start, const unsigned long long* nb_p,
-                                 unsigned long long* key, uint32_t* id, uint64_t* len, const uint4** ptr) {
+/* per sorted burst: its length (a segment's first record is a head: bursts never span segments), source start
+   (global stream index) and source pointer */
+__global__ void burst_sorted_kernel(const BucketArgs a, const uint32_t* sid, const unsigned long long* key2,
+                                    const uint64_t* start, const unsigned long long* nb_p, uint64_t* slen,
+                                    uint64_t* bsrc, const uint4** sptr) {
   const uint64_t nb = *nb_p, total = a.off[a.n_seg];
   for (uint64_t b = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; b < nb; b += (uint64_t)gridDim.x * blockDim.x) {
-    const uint64_t g = start[b];
-    const uint32_t sg = seg_of(a, g);
-    const uint4* src = a.rec[sg] + (g - a.off[sg]);
-    key[b] = ((unsigned long long)sg << a.warp_bits) | min(src->z, a.n_warps[sg]);
-    id[b] = (uint32_t)b;
-    len[b] = (b + 1 < nb ? start[b + 1] : total) - g; /* a segment's first record is a head: bursts never span */
-    ptr[b] = src;
-  }
-}
-
-__global__ void burst_sorted_kernel(const uint32_t* sid, const uint64_t* start, const uint64_t* len,
-                                    const uint4* const* ptr, const unsigned long long* nb_p, uint64_t* slen,
-                                    uint64_t* bsrc, const uint4** sptr) {
-  const uint64_t nb = *nb_p;
-  for (uint64_t b = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; b < nb; b += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t i = sid[b];
-    slen[b] = len[i];
-    bsrc[b] = start[i];
-    sptr[b] = ptr[i];
+    const uint64_t g = start[i];
+    const uint32_t sg = (uint32_t)(key2[b] >> a.warp_bits);
+    slen[b] = (i + 1 < nb ? start[i + 1] : total) - g;
+    bsrc[b] = g;
+    sptr[b] = a.rec[sg] + (g - a.off[sg]);
   }
 }
 
@@ -820,23 +824,24 @@ cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std:
   for (uint32_t i = 0; i < ns; ++i) tile0[i + 1] = tile0[i] + ((n[i] + (1u << BT_LOG) - 1) >> BT_LOG);
   const uint64_t ntile = tile0[ns];
   uint64_t* slots = (uint64_t*)alloc((ntile << BT_LOG) * 8); /* worst case: every record starts a burst */
+  unsigned long long* skey = (unsigned long long*)alloc((ntile << BT_LOG) * 8);
+  uint64_t* dtile0 = (uint64_t*)alloc((ns + 1) * 8);
   uint32_t* tile_cnt = (uint32_t*)alloc(ntile * 4 + 4);
   uint64_t* tile_cnt64 = (uint64_t*)alloc(ntile * 8 + 8);
   uint64_t* tile_off = (uint64_t*)alloc(ntile * 8 + 8);
   const uint4** drec = (const uint4**)alloc(ns * sizeof(void*));
   uint64_t* doff = (uint64_t*)alloc((ns + 1) * 8);
   uint32_t* dnw = (uint32_t*)alloc(ns * 4);
-  uint64_t* start = (uint64_t*)alloc(total * 8); /* at most one burst per record */
   unsigned long long* nb_d = (unsigned long long*)alloc(8);
-  cudaError_t e = (slots && tile_cnt && tile_cnt64 && tile_off && drec && doff && dnw && start && nb_d)
+  cudaError_t e = (slots && skey && dtile0 && tile_cnt && tile_cnt64 && tile_off && drec && doff && dnw && nb_d)
                       ? cudaSuccess : cudaErrorMemoryAllocation;
   if (e == cudaSuccess) e = cudaMemcpyAsync(drec, rec.data(), ns * sizeof(void*), cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync(doff, off.data(), (ns + 1) * 8, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync(dnw, n_warps.data(), ns * 4, cudaMemcpyHostToDevice, st);
-  for (uint32_t i = 0; i < ns && e == cudaSuccess; ++i)
-    if (n[i])
-      burst_head_kernel<<<grid_for(((n[i] + (1u << BT_LOG) - 1) >> BT_LOG) * 32, 256), 256, 0, st>>>(
-          rec[i], n[i], n_warps[i], off[i], tile0[i], slots, tile_cnt);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(dtile0, tile0.data(), (ns + 1) * 8, cudaMemcpyHostToDevice, st);
+  BucketArgs a{drec, doff, dnw, ns, warp_bits};
+  if (e == cudaSuccess && ntile)
+    burst_head_kernel<<<grid_for(ntile * 32, 256), 256, 0, st>>>(a, dtile0, ntile, slots, skey, tile_cnt);
   if (e == cudaSuccess) {
     widen_kernel<<<grid_for(ntile, 256), 256, 0, st>>>(tile_cnt, ntile, tile_cnt64);
     size_t tmp = 0;
@@ -848,22 +853,17 @@ cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std:
       if (e == cudaSuccess) e = cub::DeviceScan::InclusiveSum(dt, tmp, tile_cnt64, tile_off + 1, (int64_t)ntile, st);
     }
   }
-  if (e == cudaSuccess) {
-    burst_gather_kernel<<<grid_for(ntile * 32, 256), 256, 0, st>>>(slots, tile_cnt, tile_off, ntile, start);
-    e = cudaMemcpyAsync(nb_d, tile_off + ntile, 8, cudaMemcpyDeviceToDevice, st);
-  }
+  if (e == cudaSuccess) e = cudaMemcpyAsync(nb_d, tile_off + ntile, 8, cudaMemcpyDeviceToDevice, st);
   unsigned long long nb = 0;
   if (e == cudaSuccess) e = cudaMemcpyAsync(&nb, nb_d, 8, cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  BucketArgs a{drec, doff, dnw, ns, warp_bits};
   if (e == cudaSuccess) {
+    uint64_t* start = (uint64_t*)alloc(nb * 8 + 8);
     unsigned long long* key = (unsigned long long*)alloc(nb * 8);
     unsigned long long* key2 = (unsigned long long*)alloc(nb * 8);
     uint32_t* id = (uint32_t*)alloc(nb * 4);
     uint32_t* sid = (uint32_t*)alloc(nb * 4);
-    uint64_t* len = (uint64_t*)alloc(nb * 8);
     uint64_t* slen = (uint64_t*)alloc(nb * 8);
-    const uint4** ptr = (const uint4**)alloc(nb * sizeof(void*));
     const uint4** sptr = (const uint4**)alloc(nb * sizeof(void*));
     out->bsrc = (uint64_t*)owl_dev_alloc(nb * 8);
     out->bdst = (uint64_t*)owl_dev_alloc(nb * 8);
@@ -875,11 +875,12 @@ cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std:
       out->bk = (uint32_t*)owl_dev_alloc(nb * 4 + 4);
     }
     out->nb = nb;
-    if (!key || !key2 || !id || !sid || !len || !slen || !ptr || !sptr || !out->bsrc || !out->bdst ||
+    if (!start || !key || !key2 || !id || !sid || !slen || !sptr || !out->bsrc || !out->bdst ||
         (copy ? !out->out : (!out->bvs || !out->bpo || !out->bk)))
       e = cudaErrorMemoryAllocation;
     if (e == cudaSuccess) {
-      burst_key_kernel<<<grid_for(nb, 256), 256, 0, st>>>(a, start, nb_d, key, id, len, ptr);
+      burst_gather_kernel<<<grid_for(ntile * 32, 256), 256, 0, st>>>(slots, skey, tile_cnt, tile_off, ntile, start,
+                                                                    key, id);
       size_t tmp = 0;
       const int bits = (int)warp_bits + seg_bits;
       cub::DeviceRadixSort::SortPairs(nullptr, tmp, key, key2, id, sid, (int64_t)nb, 0, bits, st);
@@ -888,7 +889,7 @@ cudaError_t owl_bucket_segments(const std::vector<const uint4*>& rec, const std:
       else e = cub::DeviceRadixSort::SortPairs(dt, tmp, key, key2, id, sid, (int64_t)nb, 0, bits, st);
     }
     if (e == cudaSuccess) {
-      burst_sorted_kernel<<<grid_for(nb, 256), 256, 0, st>>>(sid, start, len, ptr, nb_d, slen, out->bsrc, sptr);
+      burst_sorted_kernel<<<grid_for(nb, 256), 256, 0, st>>>(a, sid, key2, start, nb_d, slen, out->bsrc, sptr);
       size_t tmp = 0;
       cub::DeviceScan::ExclusiveSum(nullptr, tmp, slen, out->bdst, (int64_t)nb, st);
       void* dt = alloc(tmp);
