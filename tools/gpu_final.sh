@@ -19,3 +19,5 @@ ncu -i ${o}_fold.ncu-rep --page source --csv --print-source cuda,sass > ${o}_fol
 python tools/ncu_lines.py ${o}_fold.src.csv 45 > ${o}_fold_lines.txt 2>&1
 rm -f ${o}_fold.src.csv
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > ${o}_smi.txt 2>&1
+timeout 900 python bench.py --channel-order --steps 5 --warmup 3 > ${o}_bench_c2_channel.json 2>${o}_bench_c2_channel.err
+timeout 900 python bench.py --channel-order --channel-mode inplace --steps 5 --warmup 3 > ${o}_bench_c2_channel_inplace.json 2>${o}_bench_c2_channel_inplace.err
