@@ -8,7 +8,7 @@ timeout 1500 python -m pytest tests -m gpu -q --timeout 900 -p no:cacheprovider 
 timeout 300 python -c "import __graft_entry__ as g; g.smoke(); print('smoke ok')" > ${o}_smoke.txt 2>&1
 timeout 900 python bench.py > ${o}_bench.json 2>${o}_bench.err
 timeout 900 python bench.py --impl reference > ${o}_bench_reference.json 2>${o}_bench_reference.err
-timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file ${o}_launches.csv \
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 6000 --csv --log-file ${o}_launches.csv \
   python bench.py --steps 1 --warmup 3 --no-cpu --no-e2e > ${o}_launches.log 2>&1
 python tools/launch_summary.py ${o}_launches.csv > ${o}_launches.txt 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:fold_kernel --launch-skip 2 -c 1 \
