@@ -74,15 +74,19 @@ def _build_full(ctx, p, channel_order=False):
     return ev[0], ev[1], n_rec
 
 
-@pytest.mark.parametrize("cfg,channel_order", [(1, False), (2, False), (3, False), (4, False), (5, False), (2, True)])
+@pytest.mark.parametrize("cfg,channel_order", [(1, False), (2, False), (3, False), (4, False), (5, False), (2, True),
+                                               (2, "inplace")])
 def test_full_size_parity(cfg, channel_order):
     """(2, True): the bench's workload in a tracer channel's order (bursts of 32, warps round-robin) gives the
-    same A-DCFGs (reading R17), through the burst bucketing."""
+    same A-DCFGs (reading R17), through the burst bucketing (copied to warp-major order, the default when it fits);
+    (2, "inplace"): the same, folded in place through the burst index (owl_config.channel_order)."""
     doc, o_ks, o_leaks = _fixture(cfg)
     p = tracegen.Params.preset(cfg)
     assert (p.runs_fix, p.runs_rnd) == (doc["runs_fix"], doc["runs_rnd"])
     ctx = api.Context(0)
-    ef, er, n_rec = _build_full(ctx, p, channel_order)
+    if channel_order == "inplace":
+        ctx.set_config(channel_order=api.OWL_CHANNEL_IN_PLACE)
+    ef, er, n_rec = _build_full(ctx, p, bool(channel_order))
     assert n_rec == doc["records"]
     bf, br = ef.export(), er.export()
     assert (len(bf), len(br)) == (doc["e_fix_bytes"], doc["e_rnd_bytes"])

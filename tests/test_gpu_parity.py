@@ -76,9 +76,9 @@ def test_malformed_same_report(ctx, variant):
     with pytest.raises(oracle.OracleError) as eo:
         oracle.build([oracle.Segment(0, 0, 0, 2, 10, rec)])
     buf = torch.from_numpy(rec.view(np.uint8).copy()).cuda()
-    for flags in (api.OWL_SEG_WARP_MAJOR, 0):
-        if variant == "mem_before_bb" and flags:
-            pass
+    # warp-major, then channel order with the bursts copied to warp-major order and folded in place
+    for flags, mode in ((api.OWL_SEG_WARP_MAJOR, 0), (0, api.OWL_CHANNEL_COPY), (0, api.OWL_CHANNEL_IN_PLACE)):
+        ctx.set_config(channel_order=mode)
         ctx.ingest([api.Segment(0, 0, 0, 2, 10, buf, len(rec), flags=flags)])
         try:
             with pytest.raises(api.OwlError, match="OWL_ERR_MALFORMED_TRACE") as eg:
@@ -86,6 +86,7 @@ def test_malformed_same_report(ctx, variant):
             assert str(eo.value).split(": ", 1)[1] in str(eg.value), (str(eo.value), str(eg.value))
         finally:
             ctx.forget_runs([0])
+            ctx.set_config()
 
 
 @pytest.mark.parametrize("cfg,div,nf,nr", [(1, 1, 10, 10), (2, 32, 3, 3), (3, 16, 2, 2), (4, 64, 2, 2), (5, 16, 3, 3)])
@@ -517,13 +518,16 @@ def test_channel_order_first_bad_record(ctx):
         oracle.build([oracle.Segment(0, 0, 0, 2, 10, rec)])
     assert f"record {early1}:" in str(eo.value)
     buf = torch.from_numpy(rec.view(np.uint8).copy()).cuda()
-    ctx.ingest([api.Segment(0, 0, 0, 2, 10, buf, len(rec), flags=0)])
-    try:
-        with pytest.raises(api.OwlError, match="OWL_ERR_MALFORMED_TRACE") as eg:
-            ctx.build([0])
-        assert str(eo.value).split(": ", 1)[1] in str(eg.value)
-    finally:
-        ctx.forget_runs([0])
+    for mode in (api.OWL_CHANNEL_COPY, api.OWL_CHANNEL_IN_PLACE):
+        ctx.set_config(channel_order=mode)
+        ctx.ingest([api.Segment(0, 0, 0, 2, 10, buf, len(rec), flags=0)])
+        try:
+            with pytest.raises(api.OwlError, match="OWL_ERR_MALFORMED_TRACE") as eg:
+                ctx.build([0])
+            assert str(eo.value).split(": ", 1)[1] in str(eg.value)
+        finally:
+            ctx.forget_runs([0])
+            ctx.set_config()
 
 
 @pytest.mark.parametrize("cfg,div,interleaved,chunk", [(2, 32, False, 0), (5, 32, True, 0), (4, 256, False, 0),
