@@ -71,14 +71,14 @@ using namespace owl_dev;
 #endif
 #define PROBE_LIMIT 4096u
 #ifndef NPAGE
-#define NPAGE 168
+#define NPAGE 160 /* with FILTER_LOG 10 the CTA's shared memory (198 KB) fits the 196 KB carve-out step (see carveout()) */
 #endif
 #define PAGE_BINS 256 /* 4-byte bins: one page counts the 1 KB address window x>>10 of one attribute */
 #ifndef DIR_LOG
 #define DIR_LOG 10
 #endif
 #ifndef FILTER_LOG
-#define FILTER_LOG 11 /* admission filter: sightings of keys not (yet) in the directory */
+#define FILTER_LOG 10 /* admission filter: sightings of keys not (yet) in the directory */
 #endif
 #define DIRCAP (1 << DIR_LOG)
 #define PAGE_TAG (3ull << 62) /* directory key lo of a page window: (x>>10) | PAGE_TAG (never a valid x) */
@@ -1037,12 +1037,20 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
 
 }  // namespace
 
+/* Preferred shared-memory carve-out (percent of the 228 KB maximum): the smallest that holds the CTA's shared memory
+   (+ the static copy of the arguments and the 1 KB the system reserves), so the rest of the 256 KB per SM is L1.
+   FoldSmem is sized to fit the 196 KB step (L1 ~60 KB instead of ~28 KB at 228 KB): +3-5% on C2 / C3 / C5
+   (profiles/r02_fold_experiments.txt #20). */
+static int carveout(size_t smem) { return (int)((smem + 2048) * 100 / (228 * 1024)); }
+
 #if FOLD_BURST
 cudaError_t owl_launch_fold_bursts(const FoldArgs& a, const FoldBurst* bursts, int grid, cudaStream_t st) {
   const size_t smem = sizeof(FoldSmem);
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(fold_burst_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(fold_burst_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, carveout(smem));
     if (e != cudaSuccess) return e;
     attr = true;
   }
@@ -1059,6 +1067,7 @@ cudaError_t owl_launch_fold(const FoldArgs& a, int grid, cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(fold_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(fold_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, carveout(smem));
     if (e != cudaSuccess) return e;
     attr = true;
   }
