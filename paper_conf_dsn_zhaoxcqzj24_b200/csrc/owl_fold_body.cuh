@@ -48,6 +48,10 @@ using namespace owl_dev;
 #ifndef FOLD_WARPS
 #define FOLD_WARPS 24 /* profiles/r01_v4_ab.txt: U2 W24 beat U1-4 x W16-32 */
 #endif
+#ifndef STEPS_IN_ST
+#define STEPS_IN_ST 1 /* the per-step accounting counter lives in the high bits of the walker's state word (bits 8..31), not in a
+                          register of its own: it was the one spill reloaded every step (profiles/r02_fold_experiments.txt #22) */
+#endif
 #ifndef FOLD_U
 #define FOLD_U 2 /* chunks of 32 records per warp and step */
 #endif
@@ -606,7 +610,11 @@ __device__ __forceinline__ void begin_traced_warp(Walker& w, RunDesc& d, const F
 #else
   w.g0 = __ldg(&w.p->z);
 #endif
+#if STEPS_IN_ST
+  w.st = (w.st & ~0xFFu) | W_INWARP; /* (bits 8..31: steps since the last accounting) */
+#else
   w.st = W_INWARP;
+#endif
   if (w.g0 >= d.n_warps) { /* every record of this warp is malformed (the first one is reported) */
     if (lane == 0) report(a.status, d.seg_index, (uint64_t)(w.p - d.rec), KERR_GWARP);
     w.st |= W_SKIP;
@@ -762,7 +770,9 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
     Walker w;
     w.p = sg.rec + first_warp_start(sg.rec, b, e, lane);
 #endif
+#if !STEPS_IN_ST
     uint32_t steps = 0; /* steps since the last accounting (a step walks <= 32 * FOLD_U records) */
+#endif
     if (lane == 0) d.p_acc = w.p;
     w.st = 0;
     w.g0 = w.cur = 0;
@@ -786,7 +796,11 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
         if (w.p >= d.tile_end) break;
         begin_traced_warp(w, d, a, lane);
       }
+#if STEPS_IN_ST
+      if ((w.st += 256u) >= (1u << 24)) { /* very long traced warp: account as we go (steps in w.st bits 8..31) */
+#else
       if (++steps >= (1u << 16)) { /* very long traced warp: account as we go */
+#endif
         __syncwarp();
         if (lane == 0) {
           const unsigned long long n = (unsigned long long)(w.p - d.p_acc);
@@ -795,7 +809,11 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
           d.p_acc = w.p;
         }
         __syncwarp();
+#if STEPS_IN_ST
+        w.st &= 0xFFu;
+#else
         steps = 0;
+#endif
         shared_on = !*(volatile unsigned int*)&s.off;
       }
       uint4 rr[FOLD_U];
