@@ -172,10 +172,12 @@ def run_reference(args):
     }), flush=True)
 
 
-def count_launches(step):
+def count_launches(step, skip=()):
     """Kernels launched by one (untimed) step, from a CUDA-activity trace: (ours, names).  'Ours' = every
     kernel compiled into libowl.so (fold / tables / KS / exchange kernels and the CUB sort kernels
-    instantiated there); torch's own memset/copy activity is not a kernel and is not counted."""
+    instantiated there); torch's own memset/copy activity is not a kernel and is not counted, nor are kernels
+    whose names contain one of `skip` (the chunked path's untimed on-device generation: tracegen's og_*
+    kernels and the torch ops around them)."""
     import torch
     from torch.profiler import ProfilerActivity, profile
     with profile(activities=[ProfilerActivity.CUDA]) as prof:
@@ -185,7 +187,7 @@ def count_launches(step):
     for ev in prof.events():
         if getattr(ev, "device_type", None) is not None and str(ev.device_type).endswith("CUDA"):
             n = ev.name
-            if n.lower().startswith(("memcpy", "memset")):
+            if n.lower().startswith(("memcpy", "memset")) or any(k in n for k in skip):
                 continue
             names[n] = names.get(n, 0) + 1
     return sum(names.values()), names
@@ -503,12 +505,9 @@ def run_ours(args):
         "result": {"n_diff_rows": out.get("n_diff"), "n_leaks": out.get("n_leaks"),
                    "cells_fix": out.get("info_f", {}).get("n_cells"), "cells_rnd": out.get("info_r", {}).get("n_cells")},
     }
-    if resident:
-        n_launch, names = count_launches(step)
-        res["gpu_launches"] = n_launch * args.steps
-        res["gpu_launches_per_step"] = names
-    else:
-        res["gpu_launches"] = None
+    n_launch, names = count_launches(step, () if resident else ("og_", "at::", "native::", "at_cuda_detail"))
+    res["gpu_launches"] = n_launch * args.steps
+    res["gpu_launches_per_step"] = names
     if not args.no_e2e:
         del segs
         ctx.forget_runs(my_runs)

@@ -5,7 +5,8 @@
  * Design v16 (the variants and their measurements: profiles/r01_v4_ab.txt, and for the round-2
  * redesign attempts profiles/r02_fold_experiments.txt).  The fold is an HBM stream whose per-record work must
  * fit the issue budget; at 24 warps per SM the register budget (80) binds, so every choice below minimises
- * instructions per 32-record chunk and live registers:
+ * instructions per 32-record chunk and live registers (what ptxas still spills stays in L1: the shared memory
+ * below fits the 196 KB carve-out, see carveout()):
  *
  *  * persistent CTAs of FOLD_WARPS independent warps; a warp pops one work item (segment, tile of 2^15
  *    records) at a time from a global counter.  A tile holds the traced warps whose first record lies in
