@@ -36,32 +36,49 @@ __global__ void clear_kernel(owl_bucket* b, uint64_t nb) {
    live keys (bits that vary across the table: the radix sort needs only those) */
 __global__ void compact_kernel(const owl_bucket* c, uint64_t cap, Key128* k, unsigned long long* cnt,
                                unsigned long long* n_out, unsigned long long* masks /* or_hi, or_lo, and_hi, and_lo */) {
+  /* each warp takes CW x 32 cells at a time and claims their output slots with ONE atomic (the table is mostly
+     empty: one atomic per 32 cells serialised on n_out) */
+  constexpr int CW = 8;
   const int lane = threadIdx.x & 31;
   unsigned long long ohi = 0, olo = 0, ahi = ~0ull, alo = ~0ull;
-  for (uint64_t base = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) & ~31ull; base < cap;
-       base += (uint64_t)gridDim.x * blockDim.x) {
-    const uint64_t i = base + lane;
-    unsigned long long vhi = OWL_EMPTY_KEY, vlo = 0, vc = 0;
-    bool live = false;
-    if (i < cap) {
-      vhi = c[i >> 1].key[i & 1][0];
-      vlo = c[i >> 1].key[i & 1][1];
-      vc = c[i >> 1].count[i & 1];
-      live = vhi != OWL_EMPTY_KEY;
+  const uint64_t step = (uint64_t)gridDim.x * blockDim.x * CW;
+  for (uint64_t base = ((blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) & ~31ull) * CW; base < cap; base += step) {
+    ulonglong2 kv[CW];
+    unsigned long long cv[CW];
+    unsigned m[CW];
+    unsigned tot = 0;
+#pragma unroll
+    for (int u = 0; u < CW; ++u) {
+      const uint64_t i = base + u * 32 + lane;
+      kv[u] = make_ulonglong2(OWL_EMPTY_KEY, 0);
+      cv[u] = 0;
+      if (i < cap) {
+        kv[u] = *reinterpret_cast<const ulonglong2*>(&c[i >> 1].key[i & 1][0]);
+        cv[u] = c[i >> 1].count[i & 1];
+      }
     }
-    const unsigned m = __ballot_sync(0xFFFFFFFFu, live);
+#pragma unroll
+    for (int u = 0; u < CW; ++u) {
+      m[u] = __ballot_sync(0xFFFFFFFFu, kv[u].x != OWL_EMPTY_KEY);
+      tot += __popc(m[u]);
+    }
+    if (!tot) continue;
     unsigned long long b = 0;
-    if (lane == 0 && m) b = atomicAdd(n_out, (unsigned long long)__popc(m));
+    if (lane == 0) b = atomicAdd(n_out, (unsigned long long)tot);
     b = __shfl_sync(0xFFFFFFFFu, b, 0);
-    if (live) {
-      const uint64_t o = b + __popc(m & ((1u << lane) - 1u));
-      k[o].hi = vhi;
-      k[o].lo = vlo;
-      cnt[o] = vc;
-      ohi |= vhi;
-      olo |= vlo;
-      ahi &= vhi;
-      alo &= vlo;
+#pragma unroll
+    for (int u = 0; u < CW; ++u) {
+      if (kv[u].x != OWL_EMPTY_KEY) {
+        const uint64_t o = b + __popc(m[u] & ((1u << lane) - 1u));
+        k[o].hi = kv[u].x;
+        k[o].lo = kv[u].y;
+        cnt[o] = cv[u];
+        ohi |= kv[u].x;
+        olo |= kv[u].y;
+        ahi &= kv[u].x;
+        alo &= kv[u].y;
+      }
+      b += __popc(m[u]);
     }
   }
   for (int o = 16; o; o >>= 1) {
