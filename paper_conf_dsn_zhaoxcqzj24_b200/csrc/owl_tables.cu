@@ -331,6 +331,66 @@ static bool pack_runs(unsigned long long mhi, unsigned long long mlo, PackRuns* 
 
 /* Canonical order of ntab tables at once (compaction, then a radix sort of the packed varying key bits,
    or of the full 128-bit keys for small tables); three host synchronisations in all. */
+/* Small tables sorted by one CTA: keys (distinct) and counts in shared memory, padded to a power of two with
+   all-ones keys, bitonic sort by (hi, lo) unsigned (the canonical order), then written out. */
+#define SMALL_SORT_MAX 4096
+namespace {
+__global__ void __launch_bounds__(1024) small_sort_kernel(const Key128* k, const unsigned long long* c, uint64_t n,
+                                                          uint32_t np2, Key128* ko, unsigned long long* co) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  Key128* sk = reinterpret_cast<Key128*>(sm);
+  unsigned long long* sc = reinterpret_cast<unsigned long long*>(sk + np2);
+  for (uint32_t i = threadIdx.x; i < np2; i += blockDim.x) {
+    if (i < n) {
+      sk[i] = k[i];
+      sc[i] = c[i];
+    } else {
+      sk[i].hi = ~0ull;
+      sk[i].lo = ~0ull;
+      sc[i] = 0;
+    }
+  }
+  __syncthreads();
+  for (uint32_t size = 2; size <= np2; size <<= 1)
+    for (uint32_t stride = size >> 1; stride; stride >>= 1) {
+      for (uint32_t t = threadIdx.x; t < np2 / 2; t += blockDim.x) {
+        const uint32_t lo = 2 * t - (t & (stride - 1)), hi = lo + stride; /* the pair (lo, hi) of this step */
+        const bool up = (lo & size) == 0;
+        const Key128 a = sk[lo], b = sk[hi];
+        const bool gt = a.hi > b.hi || (a.hi == b.hi && a.lo > b.lo);
+        if (gt == up) {
+          sk[lo] = b;
+          sk[hi] = a;
+          const unsigned long long x = sc[lo];
+          sc[lo] = sc[hi];
+          sc[hi] = x;
+        }
+      }
+      __syncthreads();
+    }
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+    ko[i] = sk[i];
+    co[i] = sc[i];
+  }
+}
+}  // namespace
+
+static cudaError_t small_sort(const Key128* k, const unsigned long long* c, uint64_t n, Key128* ko,
+                              unsigned long long* co, cudaStream_t st) {
+  uint32_t np2 = 2;
+  while (np2 < n) np2 <<= 1;
+  const size_t smem = (size_t)np2 * (sizeof(Key128) + 8);
+  static bool attr = false;
+  if (!attr) {
+    const cudaError_t e = cudaFuncSetAttribute(small_sort_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                               (int)(SMALL_SORT_MAX * (sizeof(Key128) + 8)));
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  small_sort_kernel<<<1, 1024, smem, st>>>(k, c, n, np2, ko, co);
+  return cudaGetLastError();
+}
+
 cudaError_t owl_tables_sorted(const DevTable* t, int ntab, SortedTable* out, cudaStream_t st) {
   std::vector<unsigned long long> n(ntab, 0);
   cudaError_t e = cudaSuccess;
@@ -386,6 +446,9 @@ cudaError_t owl_tables_sorted(const DevTable* t, int ntab, SortedTable* out, cud
       e = cub::DeviceRadixSort::SortPairs(dt, tmp, ck, ck2, ix, ix2, (int64_t)n[i], 0, eb, st);
       if (e == cudaSuccess)
         gather_sorted_kernel<<<grid_for(n[i], 256), 256, 0, st>>>(k0[i], c0[i], ix2, n[i], out[i].k, out[i].c);
+    } else if (n[i] <= SMALL_SORT_MAX) {
+      /* small table (the node / edge / triple tables): one CTA, bitonic in shared memory */
+      e = small_sort(k0[i], c0[i], n[i], out[i].k, out[i].c, st);
     } else {
       size_t tmp = 0;
       cub::DeviceRadixSort::SortPairs(nullptr, tmp, k0[i], out[i].k, c0[i], out[i].c, (int64_t)n[i], KeyDecomp{}, st);
