@@ -359,12 +359,19 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
         bool inplace = ctx->cfg.channel_order == OWL_CHANNEL_IN_PLACE;
         if (ctx->cfg.channel_order == OWL_CHANNEL_AUTO) {
           size_t fr = 0, tt = 0;
+          int dev = 0;
+          cudaGetDevice(&dev);
           cudaMemGetInfo(&fr, &tt);
+          fr += owl_dev_pooled(dev); /* cached blocks are reusable scratch */
           inplace = tot * 32 + (1ull << 30) > fr; /* the copy (16 B / record) next to the burst heads' scratch */
         }
         inplace = inplace && fits;
         sets.emplace_back();
+        const auto tb0 = std::chrono::steady_clock::now();
         const cudaError_t e = owl_bucket_segments(brec, bn, bw, &sets.back(), st, !inplace);
+        if (getenv("OWL_FOLD_VERBOSE"))
+          fprintf(stderr, "[owl] bucketing %s: %.3f ms (host, synchronous)\n", inplace ? "in place" : "copy",
+                  std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tb0).count());
         if (e != cudaSuccess) { status = cuda_fail(e, "fold: bucketing"); break; }
         const BucketedSet& bs = sets.back();
         for (size_t k = 0; k < bi.size(); ++k) {

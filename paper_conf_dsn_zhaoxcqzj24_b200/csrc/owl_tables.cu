@@ -169,7 +169,8 @@ int grid_for(uint64_t n, int block) {
 
 }  // namespace
 
-/* Caching device allocator: blocks are rounded up to a power of two (>= 256 B) and recycled per device,
+/* Caching device allocator: blocks are rounded up to a power of two (>= 256 B; above 1 GiB to a multiple of
+   1 GiB, so a 22 GB scratch does not hold 32 GB) and recycled per device,
    so the per-call scratch of build / sort / diff / KS never hits cudaMalloc / cudaFree (which synchronize
    the device) in steady state.  All library work of a context runs on its one stream, so a block freed
    by one call and reused by the next is ordered by that stream. */
@@ -181,7 +182,8 @@ std::map<void*, std::pair<int, size_t>> g_live;                /* block -> (devi
 
 void* owl_dev_alloc(size_t bytes) {
   size_t sz = 256;
-  while (sz < bytes) sz <<= 1;
+  if (bytes > (1ull << 30)) sz = (bytes + (1ull << 30) - 1) & ~((1ull << 30) - 1);
+  else while (sz < bytes) sz <<= 1;
   int dev = 0;
   cudaGetDevice(&dev);
   std::lock_guard<std::mutex> lk(g_pool_mu);
@@ -260,6 +262,14 @@ void owl_dev_free(void* p) {
   if (it == g_live.end()) return;
   g_pool[it->second].push_back(p);
   g_live.erase(it);
+}
+
+size_t owl_dev_pooled(int dev) {
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  size_t b = 0;
+  for (auto& f : g_pool)
+    if (f.first.first == dev) b += f.first.second * f.second.size();
+  return b;
 }
 
 void owl_dev_trim(int dev) {
