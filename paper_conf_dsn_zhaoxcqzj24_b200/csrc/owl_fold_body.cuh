@@ -52,6 +52,12 @@ using namespace owl_dev;
 #ifndef FOLD_L1PF
 #define FOLD_L1PF 1 /* prefetch each warp's next step into L1 (room for it since the 196 KB carve-out) */
 #endif
+#ifndef L1PF_STEPS
+#define L1PF_STEPS 1 /* steps ahead */
+#endif
+#ifndef L1PF_LANES
+#define L1PF_LANES 8 /* lanes 0..L1PF_LANES prefetch one 128 B line each */
+#endif
 #ifndef STEPS_IN_ST
 #define STEPS_IN_ST 1 /* the per-step accounting counter lives in the high bits of the walker's state word (bits 8..31), not in a
                           register of its own: it was the one spill reloaded every step (profiles/r02_fold_experiments.txt #22) */
@@ -844,8 +850,9 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
 #if FOLD_L1PF && !FOLD_BURST
       { /* the next step's records into L1 (lanes 0..8: one 128 B line each); the streaming loads do not allocate in
            L1 but hit what is there (profiles/r02_fold_experiments.txt #25) */
-        const char* q = (const char*)((((uintptr_t)(w.p + 32 * FOLD_U)) & ~(uintptr_t)127) + (uintptr_t)lane * 128);
-        if (lane <= 8 && q < (const char*)end) asm volatile("prefetch.global.L1 [%0];" ::"l"(q));
+        const char* q = (const char*)((((uintptr_t)(w.p + 32 * FOLD_U * L1PF_STEPS)) & ~(uintptr_t)127) +
+                                      (uintptr_t)lane * 128);
+        if (lane <= L1PF_LANES && q < (const char*)end) asm volatile("prefetch.global.L1 [%0];" ::"l"(q));
       }
 #endif
       if (!FOLD_BURST && FOLD_MODE_OF(a) != 3) { /* keep PF_DIST granules of the stream in flight to L2 */
