@@ -529,7 +529,7 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
-CHANNEL_MODES = {"auto": 0, "copy": 1, "inplace": 2}  # owl_config.channel_order
+CHANNEL_MODES = {"auto": 0, "copy": 1, "inplace": 2}  # owl_config.channel_order (auto = in place)
 
 
 def main():

@@ -111,12 +111,11 @@ typedef struct {
                                OWL_ERR_INVALID_ARG from owl_ctx_set_config.                          */
   uint32_t channel_order;   /* segments without OWL_SEG_WARP_MAJOR (a tracer channel's order, reading R17,
                                P:L183, L211) are bucketed by warp on the device, by bursts
-                               of consecutive records of one warp.  OWL_CHANNEL_AUTO (0, default): copy the
-                               bursts to a warp-major buffer when it fits in free device memory, else fold
-                               them in place; OWL_CHANNEL_COPY (1): always copy (16 B per record of
-                               scratch, the faster fold); OWL_CHANNEL_IN_PLACE (2): never copy, the fold
-                               reads every record through the burst index (needs every segment < 2^32
-                               records, else the copy is used).  Other values: OWL_ERR_INVALID_ARG.      */
+                               of consecutive records of one warp.  OWL_CHANNEL_AUTO (0, default) and
+                               OWL_CHANNEL_IN_PLACE (2): no copy, the fold reads every record through the
+                               burst index (needs every segment < 2^32 records, else the copy is used);
+                               OWL_CHANNEL_COPY (1): the bursts are copied to a warp-major buffer first
+                               (16 B per record of scratch).  Other values: OWL_ERR_INVALID_ARG.        */
 } owl_config;
 enum { OWL_CHANNEL_AUTO = 0u, OWL_CHANNEL_COPY = 1u, OWL_CHANNEL_IN_PLACE = 2u };
 

@@ -531,6 +531,11 @@ __device__ __forceinline__ void burst_window_load(Walker& w, RunDesc& d, uint64_
   d.wb = k; /* every lane writes the same values */
   d.wend = we;
   __syncwarp();
+  /* L2 prefetch of the window's bursts 1..31: the window moves on when the walk reaches its burst BURST_SLIDE, so
+     (but for the first window of a work item) every burst is prefetched at least 31 - BURST_SLIDE bursts ahead */
+  const uint32_t e = __shfl_down_sync(FULL, w.ws, 1);
+  const uint32_t end = lane == 31 ? we : e;
+  if (lane >= 1 && end > w.ws && w.ws < d.n) l2_prefetch_bulk(d.prec + w.wp, (end - w.ws) * 16u);
 }
 
 /* the window position (0..31) of the burst holding virtual record v, the window moved to start there when v + 64
@@ -553,7 +558,8 @@ __device__ __noinline__ int burst_slide(Walker& w, RunDesc& d, uint32_t v, int l
 }
 
 #ifndef BURST_SLIDE
-#define BURST_SLIDE 32 /* the window also moves once the walk reaches its BURST_SLIDE-th burst */
+#define BURST_SLIDE 24 /* the window also moves once the walk reaches its BURST_SLIDE-th burst (8 and 16 measured
+                          slower: more window loads) */
 #endif
 __device__ __forceinline__ int burst_at(Walker& w, RunDesc& d, uint32_t v, int lane) {
   const uint32_t wend = d.wend;
@@ -563,16 +569,29 @@ __device__ __forceinline__ int burst_at(Walker& w, RunDesc& d, uint32_t v, int l
   return j;
 }
 
-/* per-lane physical pointers of the step's FOLD_U chunks at virtual record v0 (nullptr at or past the segment end):
-   the burst starts inside the step are one 64-bit mask (two warp OR-reductions), a lane's burst is the one holding
-   v0 plus the starts at or before it, its start and physical offset are shuffled from the window.  Prefetches to L2
-   the burst PF_BURSTS ahead of the one holding v0. */
-#ifndef PF_BURSTS
-#define PF_BURSTS 3
-#endif
+/* per-lane physical pointers of the step's FOLD_U chunks at virtual record v0 (nullptr at or past the segment end).
+   Common case, the step within the three bursts from the one holding v0: their starts and physical offsets are
+   shuffled from the window and each lane selects.  Otherwise (shorter bursts) the burst starts inside the step are
+   one 64-bit mask (two warp OR-reductions), a lane's burst is the one holding v0 plus the starts at or before it. */
 __device__ __forceinline__ void burst_step(Walker& w, RunDesc& d, uint32_t v0, int lane, const uint4* (&q)[FOLD_U]) {
   const int j0 = burst_at(w, d, v0, lane);
   const uint32_t n = d.n, wend = d.wend;
+  { /* the step within three bursts (j0, j0 + 1, j0 + 2: bursts of at least ~21 records): a select per lane */
+    const uint32_t s0 = __shfl_sync(FULL, w.ws, j0), p0 = __shfl_sync(FULL, w.wp, j0);
+    const uint32_t a1 = __shfl_sync(FULL, w.ws, (j0 + 1) & 31), p1 = __shfl_sync(FULL, w.wp, (j0 + 1) & 31);
+    const uint32_t a2 = __shfl_sync(FULL, w.ws, (j0 + 2) & 31), p2 = __shfl_sync(FULL, w.wp, (j0 + 2) & 31);
+    const uint32_t a3 = __shfl_sync(FULL, w.ws, (j0 + 3) & 31);
+    const uint32_t e0 = j0 + 1 < 32 ? a1 : wend, e1 = j0 + 2 < 32 ? a2 : wend, e2 = j0 + 3 < 32 ? a3 : wend;
+    if (e2 >= v0 + 32 * FOLD_U || e2 >= n) {
+#pragma unroll
+      for (int u = 0; u < FOLD_U; ++u) {
+        const uint32_t t = v0 + 32 * u + lane;
+        const uint32_t off = t < e0 ? p0 + (t - s0) : (t < e1 ? p1 + (t - e0) : p2 + (t - e1));
+        q[u] = t < n ? d.prec + off : nullptr;
+      }
+      return;
+    }
+  }
   const uint32_t rel = w.ws - v0;
   const bool inb = lane > j0 && rel < 32 * FOLD_U;
   const uint32_t blo = __reduce_or_sync(FULL, inb && rel < 32 ? 1u << (rel & 31) : 0u);
@@ -599,13 +618,7 @@ __device__ __forceinline__ void burst_step(Walker& w, RunDesc& d, uint32_t v0, i
       q[u] = d.prec + __ldg(&d.bpo[lo]) + (t - __ldg(&d.bvs[lo]));
     }
   }
-  { /* L2 prefetch of a burst ahead of the walk */
-    const int jp = j0 + PF_BURSTS;
-    const uint32_t ps = __shfl_sync(FULL, w.ws, jp & 31), pp = __shfl_sync(FULL, w.wp, jp & 31);
-    const uint32_t pe = __shfl_sync(FULL, w.ws, (jp + 1) & 31);
-    const uint32_t end = jp + 1 < 32 ? pe : wend;
-    if (lane == 0 && jp < 32 && end > ps && ps < n) l2_prefetch_bulk(d.prec + pp, (end - ps) * 16u);
-  }
+
 }
 #endif
 

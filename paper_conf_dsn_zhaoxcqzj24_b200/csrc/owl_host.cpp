@@ -351,21 +351,12 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
         bi.push_back(i);
       }
       if (!bi.empty()) {
-        /* copy to a warp-major buffer (the faster fold) or walk the burst index in place (no 16 B per record of
-           scratch): owl_config.channel_order; AUTO copies when it fits with 1 GiB to spare */
-        uint64_t tot = 0;
+        /* walk the burst index in place (no 16 B per record of scratch; as fast as the copy for a tracer's bursts,
+           profiles/r02_fold_experiments.txt #27) or copy to a warp-major buffer: owl_config.channel_order; AUTO
+           folds in place whenever every segment has fewer than 2^32 records */
         bool fits = true;
-        for (uint64_t x : bn) { tot += x; fits = fits && x < (1ull << 32); }
-        bool inplace = ctx->cfg.channel_order == OWL_CHANNEL_IN_PLACE;
-        if (ctx->cfg.channel_order == OWL_CHANNEL_AUTO) {
-          size_t fr = 0, tt = 0;
-          int dev = 0;
-          cudaGetDevice(&dev);
-          cudaMemGetInfo(&fr, &tt);
-          fr += owl_dev_pooled(dev); /* cached blocks are reusable scratch */
-          inplace = tot * 32 + (1ull << 30) > fr; /* the copy (16 B / record) next to the burst heads' scratch */
-        }
-        inplace = inplace && fits;
+        for (uint64_t x : bn) fits = fits && x < (1ull << 32);
+        const bool inplace = ctx->cfg.channel_order != OWL_CHANNEL_COPY && fits;
         sets.emplace_back();
         const auto tb0 = std::chrono::steady_clock::now();
         const cudaError_t e = owl_bucket_segments(brec, bn, bw, &sets.back(), st, !inplace);

@@ -197,7 +197,6 @@ cudaError_t owl_absorb_cells(const DevTable* tabs, const ExchangeCell* cells, ui
 void* owl_dev_alloc(size_t bytes);
 void owl_dev_free(void* p);
 void owl_dev_trim(int device); /* return cached blocks to CUDA */
-size_t owl_dev_pooled(int device); /* bytes of cached (free, reusable) blocks */
 void* owl_host_alloc(size_t bytes); /* pinned (cached) host block for result rows; owl_host_free releases it */
 void owl_host_free(void* p);        /* pinned pool block or plain malloc block */
 

@@ -264,14 +264,6 @@ void owl_dev_free(void* p) {
   g_live.erase(it);
 }
 
-size_t owl_dev_pooled(int dev) {
-  std::lock_guard<std::mutex> lk(g_pool_mu);
-  size_t b = 0;
-  for (auto& f : g_pool)
-    if (f.first.first == dev) b += f.first.second * f.second.size();
-  return b;
-}
-
 void owl_dev_trim(int dev) {
   std::lock_guard<std::mutex> lk(g_pool_mu);
   for (auto& f : g_pool)

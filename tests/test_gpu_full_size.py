@@ -78,14 +78,14 @@ def _build_full(ctx, p, channel_order=False):
                                                (2, "inplace")])
 def test_full_size_parity(cfg, channel_order):
     """(2, True): the bench's workload in a tracer channel's order (bursts of 32, warps round-robin) gives the
-    same A-DCFGs (reading R17), through the burst bucketing (copied to warp-major order, the default when it fits);
-    (2, "inplace"): the same, folded in place through the burst index (owl_config.channel_order)."""
+    same A-DCFGs (reading R17), through the burst bucketing with the bursts copied to warp-major order;
+    (2, "inplace"): the same, folded in place through the burst index (owl_config.channel_order, the default)."""
     doc, o_ks, o_leaks = _fixture(cfg)
     p = tracegen.Params.preset(cfg)
     assert (p.runs_fix, p.runs_rnd) == (doc["runs_fix"], doc["runs_rnd"])
     ctx = api.Context(0)
-    if channel_order == "inplace":
-        ctx.set_config(channel_order=api.OWL_CHANNEL_IN_PLACE)
+    if channel_order:
+        ctx.set_config(channel_order=api.OWL_CHANNEL_IN_PLACE if channel_order == "inplace" else api.OWL_CHANNEL_COPY)
     ef, er, n_rec = _build_full(ctx, p, bool(channel_order))
     assert n_rec == doc["records"]
     bf, br = ef.export(), er.export()
