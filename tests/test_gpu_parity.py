@@ -249,6 +249,21 @@ def test_many_distinct_bbs(ctx):
         _build_one(ctx, over, 1)
 
 
+@pytest.mark.parametrize("n_nodes", [1, 3, 4095, 4096, 4097, 5000])
+def test_small_table_sort_boundary(ctx, n_nodes):
+    """Tables of at most 4096 cells are sorted by one CTA (bitonic in shared memory), larger ones by CUB: node /
+    edge / triple tables of sizes around the switch (distinct BB chains split over warps of <= 1000 BBs each)
+    export the oracle's canonical order."""
+    rows, b, left, w = [], 0, n_nodes, 0
+    while left:
+        k = min(left, 1000)
+        rows += [H.bb_rec(w, b + i) for i in range(k)]
+        b, left, w = b + k, left - k, w + 1
+    rec = H.to_records(rows)
+    want = oracle.build([oracle.Segment(0, 0, 0, w, 10, rec)]).export()
+    assert _build_one(ctx, rec, w) == want
+
+
 def test_wide_keys_sort_fallback(ctx):
     """More than 64 key bits vary across the address table (random 60-bit addresses, every ins and many j):
     the canonical sort takes the full 128-bit path; tables and diff still match the oracle."""
