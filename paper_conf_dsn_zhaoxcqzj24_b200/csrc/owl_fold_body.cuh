@@ -1091,6 +1091,8 @@ __global__ void __launch_bounds__(FOLD_THREADS, 1) fold_kernel(const FoldArgs ar
    FoldSmem is sized to fit the 196 KB step (L1 ~60 KB instead of ~28 KB at 228 KB): +3-5% on C2 / C3 / C5
    (profiles/r02_fold_experiments.txt #20). */
 static int carveout(size_t smem) { return (int)((smem + 2048) * 100 / (228 * 1024)); }
+static_assert(sizeof(FoldSmem) + sizeof(FoldArgs) + 1024 <= 196 * 1024,
+              "the fold's shared memory must fit the 196 KB carve-out step (else L1 shrinks to ~28 KB)");
 
 #if FOLD_BURST
 cudaError_t owl_launch_fold_bursts(const FoldArgs& a, const FoldBurst* bursts, int grid, cudaStream_t st) {
