@@ -532,10 +532,18 @@ __device__ __forceinline__ void burst_window_load(Walker& w, RunDesc& d, uint64_
   d.wend = we;
   __syncwarp();
   /* L2 prefetch of the window's bursts 1..31: the window moves on when the walk reaches its burst BURST_SLIDE, so
-     (but for the first window of a work item) every burst is prefetched at least 31 - BURST_SLIDE bursts ahead */
+     (but for the first window of a work item) every burst is prefetched at least 31 - BURST_SLIDE bursts ahead.
+     Lane l prefetches the first 5 lines of burst l (a 32-record burst), one prefetch.global.L2 per line: per-lane
+     cp.async.bulk.prefetch is serialised over the lanes. */
   const uint32_t e = __shfl_down_sync(FULL, w.ws, 1);
   const uint32_t end = lane == 31 ? we : e;
-  if (lane >= 1 && end > w.ws && w.ws < d.n) l2_prefetch_bulk(d.prec + w.wp, (end - w.ws) * 16u);
+  if (lane >= 1 && w.ws < d.n) {
+    const char* b0 = (const char*)(d.prec + w.wp);
+    const char* b1 = (const char*)(d.prec + w.wp + (end - w.ws));
+#pragma unroll
+    for (int k = 0; k < 5; ++k)
+      if (b0 + k * 128 < b1) asm volatile("prefetch.global.L2 [%0];" ::"l"(b0 + k * 128));
+  }
 }
 
 /* the window position (0..31) of the burst holding virtual record v, the window moved to start there when v + 64
