@@ -356,7 +356,9 @@ owl_status fold_pass(owl_ctx* ctx, const std::vector<PlannedSeg>& plan, DevTable
            folds in place whenever every segment has fewer than 2^32 records */
         bool fits = true;
         for (uint64_t x : bn) fits = fits && x < (1ull << 32);
-        const bool inplace = ctx->cfg.channel_order != OWL_CHANNEL_COPY && fits;
+        /* host-record waves (w >= 1) are copied: their staging buffers are reused by later waves, and a malformed
+           record's report re-reads the bucketed records after the last wave */
+        const bool inplace = ctx->cfg.channel_order != OWL_CHANNEL_COPY && fits && w == 0;
         sets.emplace_back();
         const auto tb0 = std::chrono::steady_clock::now();
         const cudaError_t e = owl_bucket_segments(brec, bn, bw, &sets.back(), st, !inplace);

@@ -545,6 +545,36 @@ def test_channel_order_first_bad_record(ctx):
             ctx.set_config()
 
 
+def test_host_records_channel_order_malformed_first_wave(ctx):
+    """Host records in channel order staged in several waves, a malformed record in the first wave: the report
+    (made after the last wave, through the bucketed records) names the oracle's record, although the first wave's
+    staging buffer has been refilled by then."""
+    ctx.set_config(host_chunk_bytes=1 << 20)
+    p = tracegen.Params.preset(2, grid_div=64, runs_fix=4, runs_rnd=0)
+    runs = list(range(p.n_runs))
+    segs, osegs = [], []
+    for r in runs:
+        for m in tracegen.run_segments(p, r):
+            rec = tracegen.interleave(tracegen.host_records(p, r, m.seq))
+            if r == 0:
+                i = int(np.flatnonzero(rec["meta"] >> 31)[5000])  # a MEM record
+                rec["addr"][i] = np.uint64(12) << np.uint64(60)
+            osegs.append(oracle.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, rec))
+            host = torch.from_numpy(rec.view(np.uint8).copy()).pin_memory()
+            segs.append(api.Segment(r, m.input_class, m.seq, m.n_warps, m.kernel_id, host, len(rec),
+                                    flags=api.OWL_SEG_HOST_RECORDS))
+    with pytest.raises(oracle.OracleError) as eo:
+        oracle.build(osegs)
+    ctx.ingest(segs)
+    try:
+        with pytest.raises(api.OwlError, match="OWL_ERR_MALFORMED_TRACE") as eg:
+            ctx.build(runs)
+        assert str(eo.value).split(": ", 1)[1] in str(eg.value), (str(eo.value), str(eg.value))
+    finally:
+        ctx.forget_runs(runs)
+        ctx.set_config()
+
+
 @pytest.mark.parametrize("cfg,div,interleaved,chunk", [(2, 32, False, 0), (5, 32, True, 0), (4, 256, False, 0),
                                                        (2, 32, False, 1 << 20), (5, 32, True, 1 << 20),
                                                        (9, 16, False, 3 << 20)])
